@@ -1,0 +1,112 @@
+// Library context: device binding, stream, stream-ordered memory pool with
+// byte accounting (peak device memory is part of the BASELINE metric), and
+// matrix storage helpers.
+#include "common.cuh"
+
+#include <cstdio>
+#include <cstring>
+
+namespace spbla {
+
+static Context g_ctx;
+Context& ctx() { return g_ctx; }
+
+void require_init() {
+    if (g_ctx.device < 0) SPBLA_THROW(SPBLA_STATUS_INVALID_STATE, "spbla_Initialize was not called");
+}
+
+void cuda_check(cudaError_t e, const char* what, const char* file, int line) {
+    if (e == cudaSuccess) return;
+    char buf[512];
+    std::snprintf(buf, sizeof(buf), "%s failed: %s (%s:%d)", what, cudaGetErrorString(e), file, line);
+    if (e == cudaErrorMemoryAllocation) {
+        (void)cudaGetLastError();
+        throw Error(SPBLA_STATUS_OUT_OF_MEMORY, buf);
+    }
+    throw Error(SPBLA_STATUS_DEVICE_ERROR, buf);
+}
+
+void check_launch(const char* name) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        char buf[256];
+        std::snprintf(buf, sizeof(buf), "kernel %s launch failed: %s", name, cudaGetErrorString(e));
+        throw Error(SPBLA_STATUS_DEVICE_ERROR, buf);
+    }
+}
+
+void* dev_alloc(size_t bytes) {
+    require_init();
+    void* p = nullptr;
+    if (bytes == 0) return nullptr;
+    cudaError_t e = cudaMallocFromPoolAsync(&p, bytes, g_ctx.pool, g_ctx.stream);
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        // give cached blocks back to the OS and retry once
+        cudaStreamSynchronize(g_ctx.stream);
+        cudaMemPoolTrimTo(g_ctx.pool, 0);
+        e = cudaMallocFromPoolAsync(&p, bytes, g_ctx.pool, g_ctx.stream);
+        if (e != cudaSuccess) {
+            (void)cudaGetLastError();
+            char buf[128];
+            std::snprintf(buf, sizeof(buf), "device allocation of %zu bytes failed", bytes);
+            throw Error(SPBLA_STATUS_OUT_OF_MEMORY, buf);
+        }
+    }
+    g_ctx.cur_bytes += bytes;
+    if (g_ctx.cur_bytes > g_ctx.peak_bytes) g_ctx.peak_bytes = g_ctx.cur_bytes;
+    return p;
+}
+
+void dev_free(void* p, size_t bytes) {
+    if (!p) return;
+    cudaFreeAsync(p, g_ctx.stream);
+    g_ctx.cur_bytes -= bytes;
+}
+
+void read_words(const uint64_t* dev, uint64_t* host, int n) {
+    CUDA_CHECK(cudaMemcpyAsync(g_ctx.host_words, dev, n * sizeof(uint64_t), cudaMemcpyDeviceToHost,
+                               g_ctx.stream));
+    CUDA_CHECK(cudaStreamSynchronize(g_ctx.stream));
+    std::memcpy(host, g_ctx.host_words, n * sizeof(uint64_t));
+}
+
+void memset_async(void* p, int v, size_t bytes) {
+    if (bytes) CUDA_CHECK(cudaMemsetAsync(p, v, bytes, g_ctx.stream));
+}
+
+void copy_async(void* dst, const void* src, size_t bytes, cudaMemcpyKind kind) {
+    if (bytes) CUDA_CHECK(cudaMemcpyAsync(dst, src, bytes, kind, g_ctx.stream));
+}
+
+void matrix_release(Matrix* m) {
+    if (m->owned) {
+        dev_free(m->rowptr, m->rowptr_cap * sizeof(off_t64));
+        dev_free(m->colidx, m->colidx_cap * sizeof(idx_t));
+    }
+    m->rowptr = nullptr;
+    m->colidx = nullptr;
+    m->rowptr_cap = m->colidx_cap = 0;
+    m->nnz = 0;
+    m->owned = true;
+}
+
+void matrix_replace(Matrix* m, off_t64* rowptr, size_t rowptr_cap, idx_t* colidx,
+                    size_t colidx_cap, uint64_t nnz) {
+    matrix_release(m);
+    m->rowptr = rowptr;
+    m->rowptr_cap = rowptr_cap;
+    m->colidx = colidx;
+    m->colidx_cap = colidx_cap;
+    m->nnz = nnz;
+    m->owned = true;
+}
+
+void matrix_set_empty(Matrix* m) {
+    DevBuf<off_t64> rp(size_t(m->nrows) + 1);
+    memset_async(rp.p, 0, rp.n * sizeof(off_t64));
+    size_t cap = rp.n;
+    matrix_replace(m, rp.detach(), cap, nullptr, 0, 0);
+}
+
+}  // namespace spbla

@@ -1,0 +1,94 @@
+// Boolean SpGEMM C (+)= A x B (§III-A l.259-264) and the
+// transitive-closure loop C += C x C (§I l.117/126).
+//
+// Step 1 (this file): the upper-bound product count per row,
+//   ub[i] = |C[i]| (accumulate) + sum_{k in A[i]} |B[k]|,
+// one 8-lane group per row (A rows average 8..32 entries in the configs),
+// coalesced colidx loads, two B row-offset loads per entry.
+// Step 2: the row engine (rowsort.cu) bins rows by ub and runs the
+// warp-bitonic / block-hash / block-bitmap kernels.
+#include "common.cuh"
+
+#include <algorithm>
+
+namespace spbla {
+
+namespace {
+
+constexpr int kGroup = 8;
+
+__global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp,
+                              const off_t64* __restrict__ crp, uint64_t* __restrict__ ub) {
+    const unsigned g = threadIdx.x & (kGroup - 1);
+    const size_t ngroups = (size_t(gridDim.x) * blockDim.x) / kGroup;
+    // warp-uniform loop: every lane of a warp runs the same trip count
+    for (size_t rb = (blockIdx.x * size_t(blockDim.x) + (threadIdx.x & ~31u)) / kGroup; rb < A.nrows;
+         rb += ngroups) {
+        const size_t r = rb + (threadIdx.x & 31) / kGroup;
+        const bool valid = r < A.nrows;
+        uint64_t s = 0;
+        if (valid) {
+            const off_t64 b = A.rowptr[r], e = A.rowptr[r + 1];
+            for (off_t64 p = b + g; p < e; p += kGroup) {
+                idx_t k = A.colidx[p];
+                s += brp[k + 1] - brp[k];
+            }
+        }
+#pragma unroll
+        for (int d = kGroup / 2; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d, kGroup);
+        if (valid && g == 0) ub[r] = s + (crp ? crp[r + 1] - crp[r] : 0);
+    }
+}
+
+}  // namespace
+
+void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
+    if (A->ncols != B->nrows || C->nrows != A->nrows || C->ncols != B->ncols)
+        SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "MxM: shapes do not conform");
+    if (!C->owned) SPBLA_THROW(SPBLA_STATUS_INVALID_ARGUMENT, "MxM: output matrix is a non-owning view");
+    const idx_t m = A->nrows;
+    if (m == 0) {
+        matrix_set_empty(C);
+        return;
+    }
+    DevBuf<uint64_t> ub(m);
+    const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
+                                                       uint64_t(ctx().num_sms) * 16);
+    const off_t64* crp = accumulate ? C->rowptr : nullptr;
+    mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, crp, ub.p);
+    count_launch();
+    check_launch("mxm_ub_kernel");
+    SegSource src{};
+    src.kind = 0;
+    src.sorted = 1;
+    src.arp = A->rowptr;
+    src.aci = A->colidx;
+    src.brp = B->rowptr;
+    src.bci = B->colidx;
+    src.crp = crp;
+    src.cci = accumulate ? C->colidx : nullptr;
+    // the engine writes fresh storage and only then installs it into C, so
+    // C may alias A and/or B
+    Matrix tmp;
+    tmp.nrows = m;
+    tmp.ncols = B->ncols;
+    row_engine(src, m, B->ncols, ub.p, &tmp);
+    matrix_replace(C, tmp.rowptr, tmp.rowptr_cap, tmp.colidx, tmp.colidx_cap, tmp.nnz);
+    tmp.rowptr = nullptr;
+    tmp.colidx = nullptr;
+}
+
+int transitive_closure(Matrix* C) {
+    if (C->nrows != C->ncols) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "closure: matrix must be square");
+    int it = 0;
+    uint64_t prev = C->nnz;
+    for (;;) {
+        mxm(C, C, C, true);
+        ++it;
+        if (C->nnz == prev) break;  // C only grows: equal nnz <=> fixed point
+        prev = C->nnz;
+    }
+    return it;
+}
+
+}  // namespace spbla
