@@ -152,7 +152,7 @@ void matrix_build(Matrix* m, const idx_t* rows, const idx_t* cols, uint64_t n, u
     Matrix tmp;
     tmp.nrows = nr;
     tmp.ncols = m->ncols;
-    row_engine(src, nr, m->ncols, cnt.p, &tmp);
+    row_engine(src, nr, m->ncols, cnt.p, nullptr, &tmp);
     matrix_replace(m, tmp.rowptr, tmp.rowptr_cap, tmp.colidx, tmp.colidx_cap, tmp.nnz);
 }
 

@@ -98,7 +98,7 @@ void transpose(Matrix* T, const Matrix* M) {
     Matrix tmp;
     tmp.nrows = nt;
     tmp.ncols = M->nrows;
-    row_engine(src, nt, M->nrows, cnt.p, &tmp);
+    row_engine(src, nt, M->nrows, cnt.p, nullptr, &tmp);
     matrix_replace(T, tmp.rowptr, tmp.rowptr_cap, tmp.colidx, tmp.colidx_cap, tmp.nnz);
 }
 

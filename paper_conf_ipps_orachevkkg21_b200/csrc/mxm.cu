@@ -17,8 +17,9 @@ namespace {
 
 constexpr int kGroup = 8;
 
-__global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp,
-                              const off_t64* __restrict__ crp, uint64_t* __restrict__ ub) {
+__global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
+                              const off_t64* __restrict__ crp, const idx_t* __restrict__ cci,
+                              uint64_t* __restrict__ ub, uint2* __restrict__ range) {
     const unsigned g = threadIdx.x & (kGroup - 1);
     const size_t ngroups = (size_t(gridDim.x) * blockDim.x) / kGroup;
     // warp-uniform loop: every lane of a warp runs the same trip count
@@ -27,8 +28,10 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp,
         const size_t r = rb + (threadIdx.x & 31) / kGroup;
         const bool valid = r < A.nrows;
         uint64_t s = 0;
+        off_t64 b = 0, e = 0;
         if (valid) {
-            const off_t64 b = A.rowptr[r], e = A.rowptr[r + 1];
+            b = A.rowptr[r];
+            e = A.rowptr[r + 1];
             for (off_t64 p = b + g; p < e; p += kGroup) {
                 idx_t k = A.colidx[p];
                 s += brp[k + 1] - brp[k];
@@ -36,7 +39,34 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp,
         }
 #pragma unroll
         for (int d = kGroup / 2; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d, kGroup);
-        if (valid && g == 0) ub[r] = s + (crp ? crp[r + 1] - crp[r] : 0);
+        if (valid && crp) s += crp[r + 1] - crp[r];
+        // column span of the row (segments are sorted: first / last entries),
+        // used by the hash and bitmap bins of the row engine
+        const bool need = valid && s > kRangeMinUb;
+        idx_t lo = 0xFFFFFFFFu, hi = 0;
+        if (need) {
+            for (off_t64 p = b + g; p < e; p += kGroup) {
+                idx_t k = A.colidx[p];
+                off_t64 x = brp[k], y = brp[k + 1];
+                if (y > x) {
+                    lo = min(lo, bci[x]);
+                    hi = max(hi, bci[y - 1]);
+                }
+            }
+            if (g == 0 && crp && crp[r + 1] > crp[r]) {
+                lo = min(lo, cci[crp[r]]);
+                hi = max(hi, cci[crp[r + 1] - 1]);
+            }
+        }
+#pragma unroll
+        for (int d = kGroup / 2; d > 0; d >>= 1) {
+            lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, d, kGroup));
+            hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, d, kGroup));
+        }
+        if (valid && g == 0) {
+            ub[r] = s;
+            if (need) range[r] = make_uint2(lo, hi);
+        }
     }
 }
 
@@ -52,10 +82,12 @@ void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
         return;
     }
     DevBuf<uint64_t> ub(m);
+    DevBuf<uint2> range(m);
     const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
                                                        uint64_t(ctx().num_sms) * 16);
     const off_t64* crp = accumulate ? C->rowptr : nullptr;
-    mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, crp, ub.p);
+    mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, crp,
+                                                  accumulate ? C->colidx : nullptr, ub.p, range.p);
     count_launch();
     check_launch("mxm_ub_kernel");
     SegSource src{};
@@ -72,7 +104,7 @@ void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
     Matrix tmp;
     tmp.nrows = m;
     tmp.ncols = B->ncols;
-    row_engine(src, m, B->ncols, ub.p, &tmp);
+    row_engine(src, m, B->ncols, ub.p, range.p, &tmp);
     matrix_replace(C, tmp.rowptr, tmp.rowptr_cap, tmp.colidx, tmp.colidx_cap, tmp.nnz);
     tmp.rowptr = nullptr;
     tmp.colidx = nullptr;

@@ -1,5 +1,5 @@
 // Row engine: per output row, the sorted duplicate-free union of a list of
-// sorted column segments, written as CSR.  This is the Gustavson row step of
+// column segments, written as CSR.  This is the Gustavson row step of
 // Boolean SpGEMM (§III-A l.259-264: nsparse-style row-wise SpGEMM;
 // for the Boolean semiring the symbolic phase IS the numeric phase, so there
 // is no value array), and the per-row sort+dedup that Build and Transpose
@@ -10,12 +10,20 @@
 //   2. scan(cap)   : scratch offsets (in-house decoupled look-back scan)
 //   3. bin_scatter : row lists per bin
 //   4. per-bin kernels, forked over 4 streams:
-//        warp bitonic (ub <= 32*E, E = 1..16): gather into smem, register
-//            bitonic sort, ballot/shuffle dedup
-//        block hash (ub <= kHashMaxUb): smem linear-probe hash, in-place
-//            compaction, smem bitonic sort
-//        block bitmap (heavier rows): smem bitmap per column window,
-//            atomicOr inserts, popc/scan emission — sorted by construction
+//        warp bitonic (ub <= 32*E, E = 1..16): flattened gather into smem,
+//            register bitonic sort, shuffle dedup
+//        block hash (ub <= 2048 / 8192): if the row's column span fits the
+//            table as a bitmap -> smem bitmap (atomicOr); else an
+//            ORDER-PRESERVING smem hash (home slot monotone in the column,
+//            linear probing without wrap-around) whose clusters are the
+//            only unsorted runs -> per-cluster insertion sort -> the table
+//            is sorted; rows whose probes run long go to the bitmap bin
+//        block bitmap (heavier rows): smem bitmap over the row's column
+//            span in windows of <= 2^20 bits, atomicOr inserts
+//      every block kernel gathers products "flattened": 32 segment
+//      descriptors per warp, lanes spread over their concatenation (shuffle
+//      binary search), 4 independent loads in flight per lane; emission is
+//      warp-chunked ballot/popc so stores are coalesced and in order.
 //   5. scan(counts): CSR row offsets
 //   6. compact     : scratch -> colidx
 #include "common.cuh"
@@ -26,12 +34,22 @@ namespace spbla {
 
 namespace {
 
-constexpr int kNumBins = 8;
-enum { BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16, BIN_HASH = 6, BIN_DENSE = 7 };
-constexpr uint64_t kHashMaxUb = 8192;      // table <= 16384 slots (64 KB smem)
-constexpr int kHashThreads = 512;
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int kNumBins = 9;
+enum { BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16, BIN_HASH_S = 6, BIN_HASH_L = 7, BIN_DENSE = 8 };
+constexpr uint64_t kWarpMaxUb = kRangeMinUb;
+constexpr uint64_t kHashSMaxUb = 2048;     // table <= 4096 slots
+constexpr uint64_t kHashLMaxUb = 8192;     // table <= 16384 slots
+constexpr int kHashSThreads = 256;
+constexpr int kHashLThreads = 512;
+constexpr uint32_t kSlack = 128;           // overflow slots past T (no wrap-around)
+constexpr uint32_t kMaxProbe = 96;
 constexpr int kDenseThreads = 1024;
-constexpr uint32_t kDenseMaxBits = 1u << 20; // 128 KB smem bitmap window
+constexpr uint32_t kDenseMaxBits = 1u << 20;  // 128 KB smem bitmap window
+constexpr int kUnroll = 4;
+constexpr uint32_t kHashSBatch = 1024;
+constexpr uint32_t kHashLBatch = 640;
+constexpr uint32_t kDenseBatch = 4096;
 
 __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub == 0) return BIN_EMPTY;
@@ -39,8 +57,9 @@ __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub <= 64) return BIN_W2;
     if (ub <= 128) return BIN_W4;
     if (ub <= 256) return BIN_W8;
-    if (ub <= 512) return BIN_W16;
-    if (ub <= kHashMaxUb) return BIN_HASH;
+    if (ub <= kWarpMaxUb) return BIN_W16;
+    if (ub <= kHashSMaxUb) return BIN_HASH_S;
+    if (ub <= kHashLMaxUb) return BIN_HASH_L;
     return BIN_DENSE;
 }
 
@@ -70,6 +89,181 @@ __device__ __forceinline__ const idx_t* get_seg(const SegSource& s, idx_t r, uin
     return s.bci + b;
 }
 
+// Flattened warp gather: every lane holds one segment (p, len); the warp
+// walks the concatenation of the 32 segments with all lanes busy and
+// kUnroll independent loads in flight per lane, calling f(q, c) for the
+// element c at concatenated position q.  Returns the total length.
+template <typename F>
+__device__ __forceinline__ uint32_t warp_flat(const idx_t* p, uint32_t len, F&& f) {
+    const unsigned lane = lane_id();
+    const uint32_t inc = warp_inclusive_scan(len);
+    const uint32_t tot = __shfl_sync(FULL, inc, 31);
+    const uint32_t exc = inc - len;
+    const unsigned long long pp = (unsigned long long)p;
+    for (uint32_t q0 = 0; q0 < tot; q0 += 32 * kUnroll) {
+        idx_t v[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            const uint32_t q = q0 + u * 32 + lane;
+            uint32_t pos = 0;  // number of lanes whose inclusive end <= q
+#pragma unroll
+            for (int st = 16; st > 0; st >>= 1) {
+                uint32_t t = __shfl_sync(FULL, inc, pos + st - 1);
+                if (t <= q) pos += st;
+            }
+            const uint32_t sl = pos > 31 ? 31 : pos;
+            const idx_t* ps = (const idx_t*)__shfl_sync(FULL, pp, sl);
+            const uint32_t es = __shfl_sync(FULL, exc, sl);
+            v[u] = q < tot ? __ldg(ps + (q - es)) : kEmpty;
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u)
+            if (v[u] != kEmpty) f(q0 + u * 32 + lane, v[u]);
+    }
+    return tot;
+}
+
+// Block-flattened gather of all products of row r:
+// segment descriptors (pointer, inclusive end) are staged in smem in batches
+// of `batch`; a block scan gives the concatenated positions; then every
+// thread takes products q = tid, tid + THREADS, ... (consecutive lanes ->
+// consecutive addresses), finds its segment by binary search in smem and
+// keeps kFlatUnroll independent loads in flight.  All warps get equal work
+// whatever the segment-length skew.
+constexpr int kFlatUnroll = 8;
+template <int THREADS, typename F>
+__device__ __forceinline__ void block_flat(const SegSource& s, idx_t r, const idx_t** sd_ptr, uint32_t* sd_end,
+                                           uint32_t batch, uint64_t* s_scan, F&& f) {
+    const uint32_t nseg = num_segs(s, r);
+    for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
+        const uint32_t n = min(batch, nseg - s0);
+        const uint32_t per = (n + THREADS - 1) / THREADS;
+        const uint32_t b = threadIdx.x * per, e = min(b + per, n);
+        uint64_t sum = 0;
+        for (uint32_t i = b; i < e; ++i) {
+            uint32_t len;
+            sd_ptr[i] = get_seg(s, r, s0 + i, len);
+            sd_end[i] = len;  // temporarily the length
+            sum += len;
+        }
+        uint64_t tot;
+        uint64_t run = block_exclusive_scan<uint64_t>(sum, s_scan, &tot);
+        for (uint32_t i = b; i < e; ++i) {
+            run += sd_end[i];
+            sd_end[i] = uint32_t(run);
+        }
+        __syncthreads();
+        const uint32_t total = uint32_t(tot);
+        for (uint32_t q0 = threadIdx.x; q0 < total; q0 += THREADS * kFlatUnroll) {
+            idx_t v[kFlatUnroll];
+#pragma unroll
+            for (int u = 0; u < kFlatUnroll; ++u) {
+                const uint32_t q = q0 + u * THREADS;
+                v[u] = kEmpty;
+                if (q < total) {
+                    uint32_t lo = 0, hi = n - 1;  // first segment whose end > q
+                    while (lo < hi) {
+                        const uint32_t mid = (lo + hi) >> 1;
+                        if (sd_end[mid] <= q) lo = mid + 1; else hi = mid;
+                    }
+                    const uint32_t st = lo ? sd_end[lo - 1] : 0u;
+                    v[u] = __ldg(sd_ptr[lo] + (q - st));
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kFlatUnroll; ++u)
+                if (v[u] != kEmpty) f(v[u]);
+        }
+        __syncthreads();  // smem descriptors are reused by the next batch
+    }
+}
+
+// Ordered, coalesced emission of the set bits of bm[0..nwords) as columns
+// base_col + 32*i + b.  Warp w owns a contiguous run of words; one block scan
+// of the per-warp counts.  Returns the count (all threads).
+__device__ __forceinline__ uint32_t emit_bitmap(const uint32_t* bm, uint32_t nwords, uint64_t base_col,
+                                                idx_t* __restrict__ out, uint32_t* s_w) {
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const uint32_t chunk = ((nwords + nw - 1) / nw + 31) & ~31u;
+    const uint32_t b = wib * chunk, e = min(b + chunk, nwords);
+    uint32_t cnt = 0;
+    for (uint32_t i = b + lane; i < e; i += 32) cnt += __popc(bm[i]);
+    cnt = warp_sum(cnt);
+    if (lane == 0) s_w[wib] = cnt;
+    __syncthreads();
+    if (wib == 0) {
+        uint32_t v = lane < nw ? s_w[lane] : 0u;
+        uint32_t inc = warp_inclusive_scan(v);
+        if (lane < nw) s_w[lane] = inc - v;
+        if (lane == nw - 1) s_w[32] = inc;
+    }
+    __syncthreads();
+    uint32_t pos = s_w[wib];
+    for (uint32_t i0 = b; i0 < e; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        uint32_t word = i < e ? bm[i] : 0u;
+        const uint32_t c = __popc(word);
+        const uint32_t inc = warp_inclusive_scan(c);
+        uint32_t o = pos + inc - c;
+        while (word) {
+            const int bit = __ffs(word) - 1;
+            word &= word - 1;
+            out[o++] = idx_t(base_col + (uint64_t(i) << 5) + bit);
+        }
+        pos += __shfl_sync(FULL, inc, 31);
+    }
+    const uint32_t total = s_w[32];
+    __syncthreads();
+    return total;
+}
+
+// Ordered, coalesced emission of an order-preserving hash table: clusters
+// (maximal runs of occupied slots) are ordered relative to each other, so an
+// element at slot i goes to  (#occupied slots before its cluster start cs)
+// + (its rank inside the cluster)  — no in-smem sort, no extra barrier.
+__device__ __forceinline__ uint32_t emit_table_ranked(const idx_t* tab, uint32_t nslots, idx_t* __restrict__ out,
+                                                      uint32_t* s_w) {
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const uint32_t chunk = ((nslots + nw - 1) / nw + 31) & ~31u;
+    const uint32_t b = wib * chunk, e = min(b + chunk, nslots);
+    uint32_t cnt = 0;
+    for (uint32_t i0 = b; i0 < e; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        cnt += __popc(__ballot_sync(FULL, i < e && tab[i] != kEmpty));
+    }
+    if (lane == 0) s_w[wib] = cnt;
+    __syncthreads();
+    if (wib == 0) {
+        uint32_t v = lane < nw ? s_w[lane] : 0u;
+        uint32_t inc = warp_inclusive_scan(v);
+        if (lane < nw) s_w[lane] = inc - v;
+        if (lane == nw - 1) s_w[32] = inc;
+    }
+    __syncthreads();
+    uint32_t pos = s_w[wib];
+    const uint32_t lt = (1u << lane) - 1u;
+    for (uint32_t i0 = b; i0 < e; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        const idx_t v = i < e ? tab[i] : kEmpty;
+        const uint32_t m = __ballot_sync(FULL, v != kEmpty);
+        if (v != kEmpty) {
+            uint32_t cs = i;
+            while (cs > 0 && tab[cs - 1] != kEmpty) --cs;
+            uint32_t rank = 0;
+            for (uint32_t j = cs; j < nslots; ++j) {
+                const idx_t w = tab[j];
+                if (w == kEmpty) break;
+                rank += (w < v);
+            }
+            out[pos + __popc(m & lt) - (i - cs) + rank] = v;
+        }
+        pos += __popc(m);
+    }
+    const uint32_t total = s_w[32];
+    __syncthreads();
+    return total;
+}
+
 // ---- 1. binning ------------------------------------------------------------
 __global__ void bin_count_kernel(const uint64_t* __restrict__ ub, idx_t nrows, idx_t ncols,
                                  uint64_t* __restrict__ cap, uint8_t* __restrict__ bin,
@@ -90,7 +284,7 @@ __global__ void bin_count_kernel(const uint64_t* __restrict__ ub, idx_t nrows, i
     if (threadIdx.x < kNumBins && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
 }
 
-// hist[0..8) -> binoff[0..9) (tiny)
+// hist[0..9) -> binoff[0..10) (tiny)
 __global__ void bin_offsets_kernel(const uint32_t* hist, uint32_t* binoff, uint32_t* cursor) {
     if (threadIdx.x == 0) {
         uint32_t s = 0;
@@ -127,31 +321,6 @@ __global__ void bin_scatter_kernel(const uint8_t* __restrict__ bin, idx_t nrows,
 }
 
 // ---- 4a. warp bitonic bins -------------------------------------------------
-// Gather all segments of row r into the warp's smem buffer; returns the count.
-__device__ __forceinline__ uint32_t warp_gather(const SegSource& s, idx_t r, idx_t* buf) {
-    const unsigned lane = lane_id();
-    const uint32_t nseg = num_segs(s, r);
-    uint32_t pos = 0;
-    for (uint32_t base = 0; base < nseg; base += 32) {
-        uint32_t j = base + lane;
-        uint32_t len = 0;
-        const idx_t* p = nullptr;
-        if (j < nseg) p = get_seg(s, r, j, len);
-        uint32_t inc = warp_inclusive_scan(len);
-        uint32_t off = pos + inc - len;
-        uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
-        uint32_t nj = min(32u, nseg - base);
-        for (uint32_t q = 0; q < nj; ++q) {
-            const idx_t* pq = (const idx_t*)__shfl_sync(0xffffffffu, (unsigned long long)p, q);
-            uint32_t lq = __shfl_sync(0xffffffffu, len, q);
-            uint32_t oq = __shfl_sync(0xffffffffu, off, q);
-            for (uint32_t t = lane; t < lq; t += 32) buf[oq + t] = __ldg(pq + t);
-        }
-        pos += tot;
-    }
-    return pos;
-}
-
 template <int E>
 __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]) {
     const unsigned lane = lane_id();
@@ -177,7 +346,7 @@ __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]) {
 #pragma unroll
                 for (int e = 0; e < E; ++e) {
                     int i = int(lane) * E + e;
-                    idx_t o = __shfl_xor_sync(0xffffffffu, x[e], lj);
+                    idx_t o = __shfl_xor_sync(FULL, x[e], lj);
                     bool lower = (i & j) == 0;
                     bool asc = (i & k) == 0;
                     x[e] = (lower == asc) ? min(x[e], o) : max(x[e], o);
@@ -199,7 +368,15 @@ warp_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
     for (uint32_t t = lo + blockIdx.x * (blockDim.x >> 5) + wib; t < hi; t += nwarps) {
         const idx_t r = rows[t];
-        uint32_t n = warp_gather(src, r, buf);
+        const uint32_t nseg = num_segs(src, r);
+        uint32_t n = 0;
+        for (uint32_t base = 0; base < nseg; base += 32) {
+            const uint32_t j = base + lane;
+            uint32_t len = 0;
+            const idx_t* p = nullptr;
+            if (j < nseg) p = get_seg(src, r, j, len);
+            n += warp_flat(p, len, [&](uint32_t q, idx_t c) { buf[n + q] = c; });
+        }
         __syncwarp();
         idx_t x[E];
 #pragma unroll
@@ -209,7 +386,7 @@ warp_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         }
         __syncwarp();
         warp_bitonic_sort<E>(x);
-        idx_t prev_last = __shfl_up_sync(0xffffffffu, x[E - 1], 1);
+        idx_t prev_last = __shfl_up_sync(FULL, x[E - 1], 1);
         uint32_t keep = 0;
         bool uniq[E];
 #pragma unroll
@@ -229,180 +406,132 @@ warp_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     }
 }
 
-// ---- 4b. block hash bin ----------------------------------------------------
+// ---- 4b. block hash / small-span bitmap bins -------------------------------
 __device__ __forceinline__ uint32_t next_pow2(uint32_t v) {
     return v <= 1 ? 1u : 1u << (32 - __clz(v - 1));
 }
 
-__global__ void __launch_bounds__(kHashThreads)
-hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ binoff,
-                const uint64_t* __restrict__ ub, idx_t* __restrict__ scratch,
-                const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
-                uint32_t* __restrict__ work) {
-    extern __shared__ idx_t tab[];
-    __shared__ uint64_t shs[33];
-    __shared__ uint32_t s_item;
-    const uint32_t lo = binoff[BIN_HASH], hi = binoff[BIN_HASH + 1];
-    const unsigned lane = lane_id(), wib = threadIdx.x >> 5, nw = blockDim.x >> 5;
+// dynamic smem: table[TMAX + kSlack] | sd_ptr[BATCH] | sd_end[BATCH]
+template <int THREADS, uint32_t TMAX, uint32_t BATCH>
+__global__ void __launch_bounds__(THREADS)
+hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
+                const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
+                idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
+                uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
+    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
+    idx_t* tab = reinterpret_cast<idx_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
+    __shared__ uint64_t s_scan[33];
+    __shared__ uint32_t s_w[33];
+    __shared__ uint32_t s_item, s_flag;
+    const uint32_t lo_i = bounds[0], hi_i = bounds[1];
     for (;;) {
-        if (threadIdx.x == 0) s_item = lo + atomicAdd(work, 1u);
+        if (threadIdx.x == 0) {
+            s_item = lo_i + atomicAdd(work, 1u);
+            s_flag = 0;
+        }
         __syncthreads();
         const uint32_t item = s_item;
-        if (item >= hi) break;
+        if (item >= hi_i) break;
         const idx_t r = rows[item];
-        const uint32_t T = next_pow2(uint32_t(2 * ub[r]));  // <= 16384
-        const uint32_t mask = T - 1;
-        const int shift = 32 - (31 - __clz(T));
-        for (uint32_t i = threadIdx.x; i < T; i += blockDim.x) tab[i] = kEmpty;
+        const uint32_t u = uint32_t(ub[r]);
+        uint32_t clo = 0, chi = ncols - 1;
+        if (range) {
+            uint2 rg = range[r];
+            clo = rg.x;
+            chi = rg.y;
+        }
+        const uint64_t span = uint64_t(chi) - clo + 1;
+        const uint32_t T = min(next_pow2(2 * u), TMAX);
+        const uint64_t words = (span + 31) >> 5;
+        const bool bitmap = words <= T;
+        const uint32_t nslots = bitmap ? uint32_t(words) : T + kSlack;
+        const idx_t fill = bitmap ? 0u : kEmpty;
+        for (uint32_t i = threadIdx.x; i < nslots; i += THREADS) tab[i] = fill;
         __syncthreads();
-        // insert: warp per segment
-        const uint32_t nseg = num_segs(src, r);
-        for (uint32_t j = wib; j < nseg; j += nw) {
-            uint32_t len;
-            const idx_t* p = get_seg(src, r, j, len);
-            for (uint32_t t = lane; t < len; t += 32) {
-                idx_t c = __ldg(p + t);
-                uint32_t h = (c * 2654435761u) >> shift;
-                if (T == 1) h = 0;
-                for (;;) {
-                    idx_t cur = tab[h];
-                    if (cur == c) break;
-                    if (cur == kEmpty) {
-                        idx_t old = atomicCAS(&tab[h], kEmpty, c);
-                        if (old == kEmpty || old == c) break;
-                    }
-                    h = (h + 1) & mask;
+        if (bitmap) {
+            block_flat<THREADS>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+                const uint32_t d = c - clo;
+                atomicOr(&tab[d >> 5], 1u << (d & 31));
+            });
+            const uint32_t n = emit_bitmap(tab, nslots, clo, scratch + soff[r], s_w);
+            if (threadIdx.x == 0) counts[r] = n;
+            continue;  // emit_bitmap ends with a barrier
+        }
+        // order-preserving home slot: floor((c - clo) * T / span) via a
+        // 32.32 fixed-point scale; monotone in c and < T
+        const uint64_t scale = (uint64_t(T) << 32) / span;
+        block_flat<THREADS>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+            uint32_t h = uint32_t((uint64_t(c - clo) * scale) >> 32);
+            for (uint32_t probe = 0;; ++probe) {
+                const idx_t cur = tab[h];
+                if (cur == c) break;
+                if (cur == kEmpty) {
+                    const idx_t old = atomicCAS(&tab[h], kEmpty, c);
+                    if (old == kEmpty || old == c) break;
+                }
+                if (++h >= nslots || probe >= kMaxProbe) {
+                    s_flag = 1;  // long cluster: hand the row to the bitmap bin
+                    break;
                 }
             }
+        });
+        // block_flat ends with a barrier
+        if (s_flag) {
+            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            __syncthreads();  // everyone has read s_flag / s_item before reuse
+            continue;
         }
-        __syncthreads();
-        // in-place compaction: each thread owns T/blockDim consecutive slots
-        const uint32_t per = T >= blockDim.x ? T / blockDim.x : 1u;
-        const uint32_t beg = threadIdx.x * per;
-        idx_t v[32];
-        uint64_t cnt = 0;
-#pragma unroll
-        for (int i = 0; i < 32; ++i) {
-            v[i] = kEmpty;
-            if (uint32_t(i) < per && beg + i < T) v[i] = tab[beg + i];
-            cnt += (v[i] != kEmpty);
-        }
-        uint64_t total;
-        uint64_t ex = block_exclusive_scan<uint64_t>(cnt, shs, &total);  // has syncs
-        uint32_t o = uint32_t(ex);
-#pragma unroll
-        for (int i = 0; i < 32; ++i)
-            if (v[i] != kEmpty) tab[o++] = v[i];
-        const uint32_t n = uint32_t(total);
-        const uint32_t N = next_pow2(n);
-        for (uint32_t i = n + threadIdx.x; i < N; i += blockDim.x) tab[i] = kEmpty;
-        __syncthreads();
-        // bitonic sort of tab[0..N)
-        for (uint32_t k = 2; k <= N; k <<= 1) {
-            for (uint32_t j = k >> 1; j > 0; j >>= 1) {
-                for (uint32_t i = threadIdx.x; i < N / 2; i += blockDim.x) {
-                    uint32_t a = 2 * j * (i / j) + (i % j);
-                    uint32_t b = a + j;
-                    bool asc = (a & k) == 0;
-                    idx_t x = tab[a], y = tab[b];
-                    if ((x > y) == asc) { tab[a] = y; tab[b] = x; }
-                }
-                __syncthreads();
-            }
-        }
-        idx_t* out = scratch + soff[r];
-        for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) out[i] = tab[i];
+        const uint32_t n = emit_table_ranked(tab, nslots, scratch + soff[r], s_w);
         if (threadIdx.x == 0) counts[r] = n;
-        __syncthreads();
     }
 }
 
 // ---- 4c. block bitmap bin ----------------------------------------------------
-__device__ __forceinline__ uint32_t lower_bound_u32(const idx_t* p, uint32_t len, idx_t key) {
-    uint32_t lo = 0, hi = len;
-    while (lo < hi) {
-        uint32_t mid = (lo + hi) >> 1;
-        if (__ldg(p + mid) < key) lo = mid + 1; else hi = mid;
-    }
-    return lo;
-}
-
+// dynamic smem: bitmap[kDenseMaxBits/32] | sd_ptr[kDenseBatch] | sd_end[kDenseBatch]
 __global__ void __launch_bounds__(kDenseThreads)
-dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ binoff,
-                 idx_t ncols, uint32_t wbits, idx_t* __restrict__ scratch,
-                 const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
-                 uint32_t* __restrict__ work) {
-    extern __shared__ uint32_t bm[];
-    __shared__ uint64_t shs[33];
+dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
+                 const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
+                 const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts, uint32_t* __restrict__ work) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
+    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + kDenseBatch * sizeof(void*));
+    uint32_t* bm = reinterpret_cast<uint32_t*>(smem_raw + kDenseBatch * (sizeof(void*) + sizeof(uint32_t)));
+    __shared__ uint64_t s_scan[33];
+    __shared__ uint32_t s_w[33];
     __shared__ uint32_t s_item;
-    const uint32_t lo = binoff[BIN_DENSE], hi = binoff[BIN_DENSE + 1];
-    const unsigned lane = lane_id(), wib = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const uint32_t wwords = wbits >> 5;
-    const uint32_t nwin = uint32_t((uint64_t(ncols) + wbits - 1) / wbits);
     for (;;) {
-        if (threadIdx.x == 0) s_item = lo + atomicAdd(work, 1u);
+        if (threadIdx.x == 0) s_item = bounds[0] + atomicAdd(work, 1u);
         __syncthreads();
         const uint32_t item = s_item;
-        if (item >= hi) break;
+        if (item >= bounds[1]) break;
         const idx_t r = rows[item];
-        const uint32_t nseg = num_segs(src, r);
-        idx_t* out = scratch + soff[r];
-        uint64_t written = 0;
-        for (uint32_t w = 0; w < nwin; ++w) {
-            const uint64_t wlo = uint64_t(w) * wbits;
-            const uint64_t whi = wlo + wbits;
-            for (uint32_t i = threadIdx.x; i < wwords; i += blockDim.x) bm[i] = 0;
-            __syncthreads();
-            for (uint32_t j = wib; j < nseg; j += nw) {
-                uint32_t len;
-                const idx_t* p = get_seg(src, r, j, len);
-                uint32_t b = 0, e = len;
-                if (nwin > 1 && !src.sorted) {
-                    // unsorted bucket: filter every element by window
-                    for (uint32_t t = lane; t < len; t += 32) {
-                        idx_t cc = __ldg(p + t);
-                        if (cc >= wlo && cc < whi) {
-                            uint32_t c = uint32_t(cc - wlo);
-                            atomicOr(&bm[c >> 5], 1u << (c & 31));
-                        }
-                    }
-                    continue;
-                }
-                if (nwin > 1) {
-                    if (lane == 0) {
-                        b = lower_bound_u32(p, len, idx_t(wlo));
-                        e = whi >= ncols ? len : lower_bound_u32(p, len, idx_t(whi));
-                    }
-                    b = __shfl_sync(0xffffffffu, b, 0);
-                    e = __shfl_sync(0xffffffffu, e, 0);
-                }
-                for (uint32_t t = b + lane; t < e; t += 32) {
-                    uint32_t c = uint32_t(__ldg(p + t) - wlo);
-                    atomicOr(&bm[c >> 5], 1u << (c & 31));
-                }
-            }
-            __syncthreads();
-            // emission: thread owns a contiguous run of words
-            const uint32_t per = (wwords + blockDim.x - 1) / blockDim.x;
-            const uint32_t beg = threadIdx.x * per;
-            const uint32_t end = min(beg + per, wwords);
-            uint64_t cnt = 0;
-            for (uint32_t i = beg; i < end; ++i) cnt += __popc(bm[i]);
-            uint64_t total;
-            uint64_t ex = block_exclusive_scan<uint64_t>(cnt, shs, &total);
-            idx_t* o = out + written + ex;
-            for (uint32_t i = beg; i < end; ++i) {
-                uint32_t word = bm[i];
-                while (word) {
-                    int bit = __ffs(word) - 1;
-                    word &= word - 1;
-                    *o++ = idx_t(wlo + (uint64_t(i) << 5) + bit);
-                }
-            }
-            written += total;
-            __syncthreads();
+        uint32_t clo = 0, chi = ncols - 1;
+        if (range) {
+            uint2 rg = range[r];
+            clo = rg.x;
+            chi = rg.y;
         }
-        if (threadIdx.x == 0) counts[r] = uint32_t(written);
+        const uint64_t span = uint64_t(chi) - clo + 1;
+        const uint32_t nwin = uint32_t((span + kDenseMaxBits - 1) / kDenseMaxBits);
+        idx_t* out = scratch + soff[r];
+        uint32_t written = 0;
+        for (uint32_t w = 0; w < nwin; ++w) {
+            const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseMaxBits;
+            const uint64_t whi = min(wlo + kDenseMaxBits, uint64_t(chi) + 1);
+            const uint32_t nwords = uint32_t((whi - wlo + 31) >> 5);
+            for (uint32_t i = threadIdx.x; i < nwords; i += blockDim.x) bm[i] = 0;
+            __syncthreads();
+            block_flat<kDenseThreads>(src, r, sd_ptr, sd_end, kDenseBatch, s_scan, [&](idx_t c) {
+                if (c >= wlo && c < whi) {
+                    const uint32_t d = uint32_t(c - wlo);
+                    atomicOr(&bm[d >> 5], 1u << (d & 31));
+                }
+            });
+            written += emit_bitmap(bm, nwords, wlo, out + written, s_w);
+        }
+        if (threadIdx.x == 0) counts[r] = written;
     }
 }
 
@@ -430,6 +559,13 @@ struct AuxStreams {
 };
 static AuxStreams g_aux;
 
+constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
+constexpr size_t kHashSSmem = (2 * kHashSMaxUb + kSlack) * sizeof(idx_t) + kHashSBatch * kSegBytes;
+constexpr size_t kHashLSmem = (2 * kHashLMaxUb + kSlack) * sizeof(idx_t) + kHashLBatch * kSegBytes;
+constexpr size_t kDenseSmem = kDenseMaxBits / 8 + kDenseBatch * kSegBytes;
+#define HASH_S hash_bin_kernel<kHashSThreads, 2 * kHashSMaxUb, kHashSBatch>
+#define HASH_L hash_bin_kernel<kHashLThreads, 2 * kHashLMaxUb, kHashLBatch>
+
 static void ensure_aux() {
     if (g_aux.device == ctx().device) return;
     for (int i = 0; i < 3; ++i) {
@@ -437,35 +573,33 @@ static void ensure_aux() {
         CUDA_CHECK(cudaEventCreateWithFlags(&g_aux.join[i], cudaEventDisableTiming));
     }
     CUDA_CHECK(cudaEventCreateWithFlags(&g_aux.fork, cudaEventDisableTiming));
-    static bool attr_done = false;
-    if (!attr_done) {
-        CUDA_CHECK(cudaFuncSetAttribute(hash_bin_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        int(2 * kHashMaxUb * sizeof(idx_t))));
-        CUDA_CHECK(cudaFuncSetAttribute(dense_bin_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        int(kDenseMaxBits / 8)));
-        attr_done = true;
-    }
+    CUDA_CHECK(cudaFuncSetAttribute(HASH_S, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kHashSSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH_L, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kHashLSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(dense_bin_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDenseSmem)));
     g_aux.device = ctx().device;
 }
 
-void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, Matrix* out) {
+void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, const uint2* range,
+                Matrix* out) {
     cudaStream_t st = ctx().stream;
     const int nsm = ctx().num_sms;
-    if (nrows == 0) {
+    if (nrows == 0 || ncols == 0) {
         matrix_set_empty(out);
         return;
     }
     ensure_aux();
     // 1. bins
-    DevBuf<uint64_t> cap(size_t(nrows) + 1);  // reused later for soff (scan in place is not allowed)
+    DevBuf<uint64_t> cap(size_t(nrows) + 1);
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    DevBuf<uint32_t> meta(64);  // hist[8] binoff[9] cursor[8] work[2]
+    // meta: hist[9] binoff[10] cursor[9] work[4] ovf[2]
+    DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
-    uint32_t* binoff = meta.p + 8;
-    uint32_t* cursor = meta.p + 17;
-    uint32_t* work = meta.p + 25;
+    uint32_t* binoff = meta.p + 10;
+    uint32_t* cursor = meta.p + 21;
+    uint32_t* work = meta.p + 31;
+    uint32_t* ovf = meta.p + 36;  // ovf[0] = 0 (list start), ovf[1] = count
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
     const unsigned gb = (unsigned)std::min<uint64_t>(ceil_div(nrows, 256), uint64_t(nsm) * 8);
     bin_count_kernel<<<gb, 256, 0, st>>>(ub, nrows, ncols, cap.p, bin.p, counts.p, hist);
@@ -484,24 +618,29 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     cap.release();
     bin.release();
     DevBuf<idx_t> scratch(scratch_total);
+    DevBuf<idx_t> ovf_rows(nrows);
 
     // 4. per-bin kernels on forked streams
     CUDA_CHECK(cudaEventRecord(g_aux.fork, st));
     for (int i = 0; i < 3; ++i) CUDA_CHECK(cudaStreamWaitEvent(g_aux.s[i], g_aux.fork, 0));
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
     {
-        cudaStream_t s3 = g_aux.s[2];  // heaviest first: dense bin
-        uint32_t wbits = kDenseMaxBits;
-        uint64_t ncr = (uint64_t(ncols) + 31) & ~uint64_t(31);
-        if (ncr < wbits) wbits = uint32_t(ncr);
-        dense_bin_kernel<<<nsm, kDenseThreads, wbits / 8, s3>>>(src, rows.p, binoff, ncols, wbits,
-                                                                scratch.p, soff.p, counts.p, work);
+        cudaStream_t s3 = g_aux.s[2];  // heaviest first
+        dense_bin_kernel<<<nsm, kDenseThreads, kDenseSmem, s3>>>(
+            src, rows.p, binoff + BIN_DENSE, range, ncols, scratch.p, soff.p, counts.p, work);
         count_launch();
         check_launch("dense_bin_kernel");
         cudaStream_t s2 = g_aux.s[1];
-        hash_bin_kernel<<<nsm * 3, kHashThreads, 2 * kHashMaxUb * sizeof(idx_t), s2>>>(
-            src, rows.p, binoff, ub, scratch.p, soff.p, counts.p, work + 1);
-        count_launch();
+        HASH_L<<<nsm * 3, kHashLThreads, kHashLSmem, s2>>>(
+            src, rows.p, binoff + BIN_HASH_L, ub, range, ncols, scratch.p, soff.p, counts.p, work + 1,
+            ovf_rows.p, ovf);
+        HASH_S<<<nsm * 7, kHashSThreads, kHashSSmem, s2>>>(
+            src, rows.p, binoff + BIN_HASH_S, ub, range, ncols, scratch.p, soff.p, counts.p, work + 2,
+            ovf_rows.p, ovf);
+        // rows whose hash probes ran long: bitmap path
+        dense_bin_kernel<<<nsm, kDenseThreads, kDenseSmem, s2>>>(
+            src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 3);
+        count_launch(3);
         check_launch("hash_bin_kernel");
         cudaStream_t s1 = g_aux.s[0];
         warp_bin_kernel<16><<<gw, 256, 0, s1>>>(src, rows.p, binoff, BIN_W16, scratch.p, soff.p, counts.p);
