@@ -1,0 +1,398 @@
+"""Benchmark of the SPbLA B200 hot path: Boolean SpGEMM C = A.A (BASELINE.json).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl b200|reference]
+
+One step = one full MxM (upper-bound pass, binning, all bin kernels,
+compaction) on the workload resident in HBM; at N > 1 (torchrun, one rank
+per GPU) a step also all-gathers the row-partitioned B over NCCL first.
+Prints ONE JSON line (rank 0).  Inputs are seeded synthetic R-MAT graphs
+(DESIGN.md §3); A (0.5 GB at the default size) is larger than L2 and a 256 MB
+buffer is also written between timed steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import spgen  # noqa: E402
+
+METRIC = "Boolean SpGEMM A·A ms & GProducts/s, HBM GB/s vs peak, peak mem @1/2/4/8 B200"
+UNIT = "GProducts/s"
+
+# BASELINE.json configs; R-MAT (a, b, c) and the reading behind each choice
+# are in DESIGN.md §3.
+WORKLOADS = {
+    "rmat22_ef32": dict(config="configs[4]", scale=22, ef=32, abc=(0.40, 0.20, 0.20), seed=5),
+    "rmat20_ef16": dict(config="configs[1]", scale=20, ef=16, abc=(0.45, 0.22, 0.22), seed=1),
+    "uniform4096": dict(config="configs[0]", scale=12, ef=8, abc=None, seed=1),
+}
+DEFAULT_WORKLOAD = "rmat22_ef32"
+FLUSH_BYTES = 256 << 20
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def gen_pairs(wl, device):
+    n = 1 << wl["scale"]
+    if wl["abc"] is None:
+        r, c = spgen.uniform_pairs(n, n, wl["ef"], wl["seed"], device=device)
+    else:
+        r, c = spgen.rmat_pairs(wl["scale"], wl["ef"], *wl["abc"], seed=wl["seed"], device=device)
+    return n, r, c
+
+
+def row_products(rowptr, colidx, n):
+    """Per-row product count sum_{k in A[i]} |B[k]| (B = A), planning only."""
+    lens = rowptr[1:] - rowptr[:-1]
+    rows = torch.repeat_interleave(torch.arange(n, device=rowptr.device), lens)
+    ub = torch.zeros(n, dtype=torch.int64, device=rowptr.device)
+    ub.index_add_(0, rows, lens[colidx.long()])
+    return ub, rows
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.proc = None
+        self.out = None
+        try:
+            self.out = open(f"/tmp/clocks_{os.getpid()}.csv", "w+")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(gpu_index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=self.out, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.out.seek(0)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in self.out.read().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        self.out.close()
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+def cpu_oracle_sample(rp_host, ci_host, ub_host, target_products):
+    """Time the CPU oracle (as it stands) on every k-th row of the workload."""
+    import numpy as np
+    import oracle
+    n = len(rp_host) - 1
+    total = int(ub_host.sum())
+    k = max(1, int(np.ceil(total / target_products)))
+    rows = np.arange(0, n, k, dtype=np.uint32)
+    prods = int(ub_host[rows.astype(np.int64)].sum())
+    A = oracle.Csr(n, n, rp_host, ci_host)
+    t = time.perf_counter()
+    out = oracle.mxm_rows(A, A, rows)
+    dt = time.perf_counter() - t
+    return prods, dt, len(rows), k, out.nvals
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, bounded sample per step."""
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if rank != 0:
+        return
+    import numpy as np
+    wl = WORKLOADS[args.workload]
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    n, r, c = gen_pairs(wl, dev)
+    # setup only (untimed): sorted duplicate-free CSR with plain torch ops
+    key = torch.unique(r.long() * n + c.long())
+    rows = key // n
+    ci = (key % n).to(torch.int32)
+    rp = torch.zeros(n + 1, dtype=torch.int64, device=key.device)
+    rp[1:] = torch.cumsum(torch.bincount(rows, minlength=n), 0)
+    del r, c, key, rows
+    ub, _ = row_products(rp, ci, n)
+    rp_h = rp.cpu().numpy().astype(np.uint64)
+    ci_h = ci.cpu().numpy().astype(np.uint32)
+    ub = ub.cpu().numpy()
+    target = float(os.environ.get("REF_SAMPLE_PRODUCTS", "3e7"))
+    times, prods = [], 0
+    for i in range(args.warmup + args.steps):
+        p, dt, nrows, k, _ = cpu_oracle_sample(rp_h, ci_h, ub, target)
+        if i >= args.warmup:
+            times.append(dt)
+            prods = p
+    ms = 1e3 * sum(times) / len(times)
+    value = prods / (ms * 1e-3) / 1e9
+    sample = f"every {k}-th row ({nrows} rows, {prods} products) of {args.workload}, std::set Gustavson, 1 thread"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": args.workload, "baseline_config": wl["config"]},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default=DEFAULT_WORKLOAD, choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    args.warmup = max(args.warmup, 3)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    import torch.distributed as dist
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    import paper_conf_ipps_orachevkkg21_b200 as sp
+    from paper_conf_ipps_orachevkkg21_b200 import dist as spdist
+    sp.Initialize(local)
+    stream = torch.cuda.current_stream()
+    wl = WORKLOADS[args.workload]
+
+    # ---- setup (untimed): generate, build, plan --------------------------------
+    t0 = time.time()
+    n, r, c = gen_pairs(wl, "cuda")
+    Afull = sp.Matrix.from_pairs(n, n, r, c)
+    del r, c
+    rp_full, ci_full = Afull.device_tensors()
+    ub_full, _ = row_products(rp_full, ci_full, n)
+    if world > 1:
+        bounds = spdist.product_balanced_bounds(ub_full, world)
+    else:
+        bounds = [0, n]
+    r0, r1 = bounds[rank], bounds[rank + 1]
+    if world > 1:
+        A = sp.submatrix(Afull, r0, 0, r1 - r0, n)  # this rank's rows of A (and of B = A)
+        del rp_full, ci_full
+        Afull.free()
+        ops = spdist.CudaOps(sp)
+    else:
+        A = Afull
+    ub = ub_full[r0:r1]
+    products_local = int(ub.sum())
+    prod_t = torch.tensor([products_local], dtype=torch.int64, device="cuda")
+    if world > 1:
+        dist.all_reduce(prod_t)
+    products = int(prod_t)
+    nnzA = A.nvals
+    log(f"[rank {rank}] setup {time.time() - t0:.1f}s: n={n} rows[{r0},{r1}) nnzA={nnzA} "
+        f"products(total)={products}")
+
+    C = sp.Matrix.new(r1 - r0, n)
+
+    def step():
+        if world > 1:
+            return spdist.distributed_mxm(ops, A, A, n, n, C_local=C)
+        sp.MxM(C, A, A)
+        return C
+
+    flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device="cuda")
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    nnzC_local = C.nvals
+
+    # ---- timed region ------------------------------------------------------------
+    sp.reset_peak_memory()
+    sp.reset_launch_count()
+    if not os.environ.get("BENCH_NO_KTIME"):
+        sp.set_kernel_timing(True)
+    clocks = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    step_ms = []
+    for _ in range(args.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        step()
+        e1.record(stream)
+        e1.synchronize()
+        step_ms.append(e0.elapsed_time(e1))
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    log(f"[rank {rank}] step ms: {[round(x, 2) for x in step_ms]}")
+    launches = sp.launch_count()
+    ktimes = {k: sp.kernel_timing(k) for k in
+              ("mxm_ub", "warp_bins", "hash_s", "hash_l", "hash_x", "dense", "compact")}
+    sp.set_kernel_timing(False)
+    peak_mem = sp.memory_stats()[1]
+    tot = torch.tensor([sum(step_ms), peak_mem, nnzC_local, launches], dtype=torch.float64, device="cuda")
+    if world > 1:
+        mx = tot.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        sm = tot.clone()
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        total_ms, peak_mem_max = float(mx[0]), float(mx[1])
+        nnzC, launches_all = int(sm[2]), int(sm[3])
+    else:
+        total_ms, peak_mem_max, nnzC, launches_all = float(tot[0]), float(tot[1]), int(tot[2]), int(tot[3])
+    ms = total_ms / args.steps
+    value = products / (ms * 1e-3) / 1e9
+
+    # ---- roofline of the dominant kernel (rank-local, reported by rank 0) ---
+    thr = sp.engine_thresholds()
+    peak_gbs, peak_src = load_peaks()
+    roof = None
+    dom = max(("warp_bins", "hash_s", "hash_l", "hash_x", "dense"), key=lambda k: ktimes[k][0])
+    dms, dn = ktimes[dom]
+    if dn:
+        rp_a, ci_a = A.device_tensors()
+        crp, _ = C.device_tensors()
+        lens_a = (rp_a[1:] - rp_a[:-1])
+        outs = (crp[1:] - crp[:-1])
+        lo_hi = {"warp_bins": (0, thr[4]), "hash_s": (thr[4], thr[5]), "hash_l": (thr[5], thr[6]),
+                 "hash_x": (thr[6], thr[7]), "dense": (thr[7], 1 << 62)}[dom]
+        sel = (ub > lo_hi[0]) & (ub <= lo_hi[1])
+        seg = int(lens_a[sel].sum())
+        prod_b = int(ub[sel].sum())
+        out_b = int(outs[sel].sum())
+        rows_b = int(sel.sum())
+        # algorithmic bytes: 4 B per gathered product, 20 B per
+        # segment descriptor (A colidx + B row-offset pair), 4 B per output
+        # column written, 32 B per row of per-row metadata
+        alg_bytes = 4 * prod_b + 20 * seg + 4 * out_b + 32 * rows_b
+        per_launch_ms = dms / dn
+        achieved = alg_bytes / (per_launch_ms * 1e-3) / 1e9
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        if os.path.exists(tp):
+            with open(tp) as f:
+                tj = json.load(f)
+            traffic = tj.get(args.workload, {}).get(dom)
+        roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak_gbs, "unit": "GB/s",
+                "frac": achieved / peak_gbs, "traffic": traffic, "alg_bytes_per_launch": alg_bytes,
+                "launch_ms": per_launch_ms, "peak_source": peak_src,
+                "kernel_ms_per_step": {k: v[0] / max(1, args.steps) for k, v in ktimes.items()}}
+
+    # ---- e2e through the C ABI with host buffers --------------------------------
+    e2e = None
+    if not args.no_e2e:
+        rp_h = torch.empty(A.nrows + 1, dtype=torch.int64).pin_memory()
+        ci_h = torch.empty(max(nnzA, 1), dtype=torch.int32).pin_memory()
+        A.export_csr(rp_h, ci_h[:nnzA])
+        crp_h = torch.empty(C.nrows + 1, dtype=torch.int64).pin_memory()
+        cci_h = torch.empty(max(nnzC_local, 1), dtype=torch.int32).pin_memory()
+        Ae = sp.Matrix.new(A.nrows, n)
+        Ce = sp.Matrix.new(C.nrows, n)
+        e2e_steps = min(args.steps, 3)
+        e2e_ms = []
+        h2d = (A.nrows + 1) * 8 + nnzA * 4
+        d2h = (C.nrows + 1) * 8 + nnzC_local * 4
+        for i in range(e2e_steps + 1):
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            Ae.import_csr(rp_h, ci_h[:nnzA])
+            if world > 1:
+                spdist.distributed_mxm(ops, Ae, Ae, n, n, C_local=Ce)
+            else:
+                sp.MxM(Ce, Ae, Ae)
+            Ce.export_csr(crp_h, cci_h[:nnzC_local])
+            torch.cuda.synchronize()
+            if i:
+                e2e_ms.append(1e3 * (time.perf_counter() - t))
+        et = torch.tensor([sum(e2e_ms) / len(e2e_ms)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e2e = {"value": products / (float(et) * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": float(et), "steps": e2e_steps,
+               "path": "ImportCSR(pinned host) -> MxM -> ExportCSR(pinned host)"}
+        Ae.free()
+        Ce.free()
+
+    # ---- CPU oracle baseline (rank 0, N = 1) --------------------------------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        rp_h, ci_h = A.to_csr()
+        p, dt, nr_s, k, _ = cpu_oracle_sample(rp_h, ci_h, ub.cpu().numpy(),
+                                              float(os.environ.get("CPU_SAMPLE_PRODUCTS", "8e7")))
+        cpu = {"value": p / dt / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"every {k}-th row ({nr_s} rows, {p} products) of {args.workload}; "
+                         f"{dt:.1f}s single-threaded std::set Gustavson"}
+
+    if rank == 0:
+        a_, b_, c_ = wl["abc"] if wl["abc"] else (None, None, None)
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic (seeded R-MAT, DESIGN.md §3)",
+            "config": {"workload": args.workload, "baseline_config": wl["config"], "rows": n,
+                       "edge_factor": wl["ef"], "rmat_abc": wl["abc"], "nnz_A": int(nnzA) if world == 1 else None,
+                       "products": products, "nnz_C": nnzC, "parallelism": f"rows{world}",
+                       "l2": "A larger than L2 (126 MB) and a 256 MB write between timed steps",
+                       "peak_mem_gb": peak_mem_max / 1e9},
+            "peak_mem_gb": peak_mem_max / 1e9,
+            "gpu_launches": launches_all,
+            "clocks": clk,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

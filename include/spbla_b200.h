@@ -19,7 +19,9 @@
  *
  * Conventions for every entry point:
  *  - Returns SPBLA_STATUS_SUCCESS (0) or an error code; on error no output
- *    matrix is modified, and spbla_GetLastErrorMessage() describes the error.
+ *    matrix is modified (exception: a failed non-accumulating MxM leaves C
+ *    empty, its old content having been released to lower the memory peak),
+ *    and spbla_GetLastErrorMessage() describes the error.
  *  - All device work is enqueued on the library stream (spbla_SetStream; the
  *    legacy default stream until set).  Entry points that must learn a result
  *    size on the host (Build, MxM, EWiseAdd, Transpose, ExtractSubMatrix,
@@ -92,6 +94,17 @@ const char* spbla_GetVersion(void);
  * bench's "gpu_launches" evidence). */
 uint64_t spbla_GetLaunchCount(void);
 void spbla_ResetLaunchCount(void);
+/* Per-kernel CUDA-event timing on each kernel's launching stream (bench.py's
+ * roofline evidence).  enable != 0 clears previous records and starts
+ * recording; spbla_GetKernelTiming sums the recorded launches of the named
+ * kernel group ("mxm_ub", "warp_bins", "hash_s", "hash_l", "hash_x", "dense",
+ * "compact") and synchronises on their end events. */
+spbla_Status spbla_SetKernelTiming(int enable);
+spbla_Status spbla_GetKernelTiming(const char* name, double* total_ms, uint64_t* launches);
+/* Upper-bound ("ub") limits of the row engine's bins, ascending: warp bins
+ * E=1,2,4,8,16, hash-small, hash-large, hash-xl; rows above the last go to
+ * the bitmap bin.  *n: capacity in, count out. */
+spbla_Status spbla_GetEngineThresholds(uint64_t* thresholds, uint32_t* n);
 
 /* ---- matrix life cycle --------------------------- */
 

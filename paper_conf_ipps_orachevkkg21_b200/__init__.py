@@ -98,6 +98,25 @@ def reset_launch_count():
     _lib().spbla_ResetLaunchCount()
 
 
+def set_kernel_timing(enable: bool):
+    _check(_lib().spbla_SetKernelTiming(1 if enable else 0), "spbla_SetKernelTiming")
+
+
+def kernel_timing(name: str):
+    """(total ms, launches) of a kernel group recorded since set_kernel_timing(True)."""
+    ms, n = ctypes.c_double(), ctypes.c_uint64()
+    _check(_lib().spbla_GetKernelTiming(name.encode(), ctypes.byref(ms), ctypes.byref(n)),
+           "spbla_GetKernelTiming")
+    return float(ms.value), int(n.value)
+
+
+def engine_thresholds():
+    buf = (ctypes.c_uint64 * 16)()
+    n = ctypes.c_uint32(16)
+    _check(_lib().spbla_GetEngineThresholds(buf, ctypes.byref(n)), "spbla_GetEngineThresholds")
+    return [int(buf[i]) for i in range(n.value)]
+
+
 def _ptr(a):
     """Raw address of a torch tensor / numpy array, and whether it is host memory."""
     if a is None:

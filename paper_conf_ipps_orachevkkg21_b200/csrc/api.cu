@@ -22,6 +22,9 @@ void matrix_duplicate(const Matrix* m, Matrix* d);
 void matrix_assemble(Matrix* m, uint32_t nblocks, const idx_t* nrows, const off_t64* const* rowptr,
                      const idx_t* const* colidx, const uint64_t* nnz);
 void validate_csr(const off_t64* rowptr, const idx_t* colidx, idx_t nrows, idx_t ncols, uint64_t nnz);
+void ktime_enable(bool on);
+void ktime_query(const char* name, double* total_ms, uint64_t* launches);
+void engine_thresholds(uint64_t* out, uint32_t* n);
 }  // namespace spbla
 
 using namespace spbla;
@@ -123,6 +126,27 @@ spbla_Status spbla_ResetPeakMemory(void) {
 const char* spbla_GetLastErrorMessage(void) { return g_last_error.c_str(); }
 const char* spbla_GetVersion(void) { return "spbla_b200 0.1 (sm_100a)"; }
 uint64_t spbla_GetLaunchCount(void) { return ctx().launches; }
+
+spbla_Status spbla_SetKernelTiming(int enable) {
+    return guarded([&] {
+        require_init();
+        ktime_enable(enable != 0);
+    });
+}
+
+spbla_Status spbla_GetKernelTiming(const char* name, double* total_ms, uint64_t* launches) {
+    return guarded([&] {
+        NEED(name && total_ms && launches, "null argument");
+        ktime_query(name, total_ms, launches);
+    });
+}
+
+spbla_Status spbla_GetEngineThresholds(uint64_t* thresholds, uint32_t* n) {
+    return guarded([&] {
+        NEED(thresholds && n, "null argument");
+        engine_thresholds(thresholds, n);
+    });
+}
 void spbla_ResetLaunchCount(void) { ctx().launches = 0; }
 
 spbla_Status spbla_Matrix_New(spbla_Matrix* matrix, spbla_Index nrows, spbla_Index ncols) {

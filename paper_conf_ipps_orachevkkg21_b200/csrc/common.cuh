@@ -50,6 +50,10 @@ void read_words(const uint64_t* dev, uint64_t* host, int n);
 void memset_async(void* p, int v, size_t bytes);
 void copy_async(void* dst, const void* src, size_t bytes, cudaMemcpyKind kind);
 inline void count_launch(int n = 1) { ctx().launches += n; }
+// Optional per-kernel CUDA-event timing on the launching stream (bench.py's
+// roofline evidence): ktime_begin returns -1 when timing is off.
+int ktime_begin(const char* name, cudaStream_t s);
+void ktime_end(int slot);
 void check_launch(const char* name);
 
 // RAII device buffer in the pool.

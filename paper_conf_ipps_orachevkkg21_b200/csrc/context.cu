@@ -5,6 +5,8 @@
 
 #include <cstdio>
 #include <cstring>
+#include <string>
+#include <vector>
 
 namespace spbla {
 
@@ -107,6 +109,59 @@ void matrix_set_empty(Matrix* m) {
     memset_async(rp.p, 0, rp.n * sizeof(off_t64));
     size_t cap = rp.n;
     matrix_replace(m, rp.detach(), cap, nullptr, 0, 0);
+}
+
+struct KRec {
+    std::string name;
+    cudaStream_t stream;
+    cudaEvent_t a, b;
+};
+static bool g_ktime_on = false;
+static std::vector<KRec> g_krec;
+static std::vector<cudaEvent_t> g_kevpool;
+static size_t g_kev_used = 0;
+
+static cudaEvent_t kev() {
+    if (g_kev_used == g_kevpool.size()) {
+        cudaEvent_t e;
+        CUDA_CHECK(cudaEventCreate(&e));
+        g_kevpool.push_back(e);
+    }
+    return g_kevpool[g_kev_used++];
+}
+
+int ktime_begin(const char* name, cudaStream_t s) {
+    if (!g_ktime_on) return -1;
+    KRec r{name, s, kev(), kev()};
+    CUDA_CHECK(cudaEventRecord(r.a, s));
+    g_krec.push_back(r);
+    return int(g_krec.size()) - 1;
+}
+
+void ktime_end(int slot) {
+    if (slot < 0) return;
+    CUDA_CHECK(cudaEventRecord(g_krec[slot].b, g_krec[slot].stream));
+}
+
+void ktime_enable(bool on) {
+    g_ktime_on = on;
+    g_krec.clear();
+    g_kev_used = 0;
+}
+
+void ktime_query(const char* name, double* total_ms, uint64_t* launches) {
+    double t = 0;
+    uint64_t n = 0;
+    for (auto& r : g_krec) {
+        if (r.name != name) continue;
+        CUDA_CHECK(cudaEventSynchronize(r.b));
+        float ms = 0;
+        CUDA_CHECK(cudaEventElapsedTime(&ms, r.a, r.b));
+        t += ms;
+        ++n;
+    }
+    *total_ms = t;
+    *launches = n;
 }
 
 }  // namespace spbla

@@ -72,11 +72,14 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
 
 }  // namespace
 
-void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
+static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
     if (A->ncols != B->nrows || C->nrows != A->nrows || C->ncols != B->ncols)
         SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "MxM: shapes do not conform");
     if (!C->owned) SPBLA_THROW(SPBLA_STATUS_INVALID_ARGUMENT, "MxM: output matrix is a non-owning view");
     const idx_t m = A->nrows;
+    // C = A x B does not read C: give its storage back to the pool before the
+    // engine allocates scratch and the result (lowers the peak by nnz(C_old))
+    if (!accumulate && C != A && C != B) matrix_release(C);
     if (m == 0) {
         matrix_set_empty(C);
         return;
@@ -86,8 +89,10 @@ void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
     const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
                                                        uint64_t(ctx().num_sms) * 16);
     const off_t64* crp = accumulate ? C->rowptr : nullptr;
+    int tk = ktime_begin("mxm_ub", ctx().stream);
     mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, crp,
                                                   accumulate ? C->colidx : nullptr, ub.p, range.p);
+    ktime_end(tk);
     count_launch();
     check_launch("mxm_ub_kernel");
     SegSource src{};
@@ -108,6 +113,22 @@ void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
     matrix_replace(C, tmp.rowptr, tmp.rowptr_cap, tmp.colidx, tmp.colidx_cap, tmp.nnz);
     tmp.rowptr = nullptr;
     tmp.colidx = nullptr;
+}
+
+void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
+    try {
+        mxm_impl(C, A, B, accumulate);
+    } catch (...) {
+        // a non-accumulating MxM may have released C already: leave it a
+        // valid empty matrix rather than a dangling one
+        if (C->rowptr == nullptr) {
+            try {
+                matrix_set_empty(C);
+            } catch (...) {
+            }
+        }
+        throw;
+    }
 }
 
 int transitive_closure(Matrix* C) {

@@ -9,47 +9,47 @@
 //   1. bin_count   : cap[r] = min(ub[r], ncols), bin[r] by ub, bin histogram
 //   2. scan(cap)   : scratch offsets (in-house decoupled look-back scan)
 //   3. bin_scatter : row lists per bin
-//   4. per-bin kernels, forked over 4 streams:
+//   4. per-bin kernels:
 //        warp bitonic (ub <= 32*E, E = 1..16): flattened gather into smem,
 //            register bitonic sort, shuffle dedup
-//        block hash (ub <= 2048 / 8192): if the row's column span fits the
-//            table as a bitmap -> smem bitmap (atomicOr); else an
-//            ORDER-PRESERVING smem hash (home slot monotone in the column,
-//            linear probing without wrap-around) whose clusters are the
-//            only unsorted runs -> per-cluster insertion sort -> the table
-//            is sorted; rows whose probes run long go to the bitmap bin
-//        block bitmap (heavier rows): smem bitmap over the row's column
-//            span in windows of <= 2^20 bits, atomicOr inserts
-//      every block kernel gathers products "flattened": 32 segment
-//      descriptors per warp, lanes spread over their concatenation (shuffle
-//      binary search), 4 independent loads in flight per lane; emission is
-//      warp-chunked ballot/popc so stores are coalesced and in order.
+//        block hash (ub <= 2048 / 8192 / 24576, 256 / 512 / 1024 threads):
+//            a smem bitmap when the row's column span fits the table, else
+//            an ORDER-PRESERVING hash (home slot monotone in the column,
+//            linear probing upward, no wrap-around): clusters are mutually
+//            ordered, so emission writes each element at (#occupied slots
+//            before its cluster) + (rank inside the cluster) - sorted output
+//            without a sort; rows whose probes run long go to the bitmap bin
+//        block bitmap (heavier rows): two-level smem bitmap over the row's
+//            column span in windows of 2^20 bits; the top level (one bit per
+//            word) makes clearing and emission proportional to touched words
+//      block kernels stage compacted segment descriptors in smem (pointer
+//      pre-offset by the segment's concatenated start, inclusive end), then
+//      each warp walks 256 consecutive products: 32 candidate segments per
+//      lane-window, shuffle binary search, 8 independent loads in flight.
 //   5. scan(counts): CSR row offsets
 //   6. compact     : scratch -> colidx
 #include "common.cuh"
 
 #include <algorithm>
+#include <cstdlib>
 
 namespace spbla {
 
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int kNumBins = 9;
-enum { BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16, BIN_HASH_S = 6, BIN_HASH_L = 7, BIN_DENSE = 8 };
-constexpr uint64_t kWarpMaxUb = kRangeMinUb;
-constexpr uint64_t kHashSMaxUb = 2048;     // table <= 4096 slots
-constexpr uint64_t kHashLMaxUb = 8192;     // table <= 16384 slots
-constexpr int kHashSThreads = 256;
-constexpr int kHashLThreads = 512;
-constexpr uint32_t kSlack = 128;           // overflow slots past T (no wrap-around)
+constexpr int kNumBins = 10;
+enum {
+    BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16,
+    BIN_HASH_S = 6, BIN_HASH_L = 7, BIN_HASH_X = 8, BIN_DENSE = 9
+};
+constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 512
+constexpr uint64_t kHashSMaxUb = 2048;
+constexpr uint64_t kHashLMaxUb = 8192;
+constexpr uint64_t kHashXMaxUb = 24576;
 constexpr uint32_t kMaxProbe = 96;
-constexpr int kDenseThreads = 1024;
-constexpr uint32_t kDenseMaxBits = 1u << 20;  // 128 KB smem bitmap window
-constexpr int kUnroll = 4;
-constexpr uint32_t kHashSBatch = 1024;
-constexpr uint32_t kHashLBatch = 640;
-constexpr uint32_t kDenseBatch = 4096;
+constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
+constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
 __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub == 0) return BIN_EMPTY;
@@ -60,6 +60,7 @@ __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub <= kWarpMaxUb) return BIN_W16;
     if (ub <= kHashSMaxUb) return BIN_HASH_S;
     if (ub <= kHashLMaxUb) return BIN_HASH_L;
+    if (ub <= kHashXMaxUb) return BIN_HASH_X;
     return BIN_DENSE;
 }
 
@@ -123,81 +124,115 @@ __device__ __forceinline__ uint32_t warp_flat(const idx_t* p, uint32_t len, F&& 
     return tot;
 }
 
-// Block-flattened gather of all products of row r:
-// segment descriptors (pointer, inclusive end) are staged in smem in batches
-// of `batch`; a block scan gives the concatenated positions; then every
-// thread takes products q = tid, tid + THREADS, ... (consecutive lanes ->
-// consecutive addresses), finds its segment by binary search in smem and
-// keeps kFlatUnroll independent loads in flight.  All warps get equal work
-// whatever the segment-length skew.
-constexpr int kFlatUnroll = 8;
-template <int THREADS, typename F>
-__device__ __forceinline__ void block_flat(const SegSource& s, idx_t r, const idx_t** sd_ptr, uint32_t* sd_end,
-                                           uint32_t batch, uint64_t* s_scan, F&& f) {
+// ---- block gather ----------------------------------------------------------
+// Stage the non-empty segments among [s0, s0+n) of row r: sd_ptr[k] points
+// at the segment minus its start offset in the concatenation (so product q
+// of segment k is sd_ptr[k][q]), sd_end[k] is its inclusive end.  Returns the
+// number of products; *ns = number of staged segments.  Ends with a barrier.
+template <int THREADS>
+__device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint32_t s0, uint32_t n,
+                                                   const idx_t** sd_ptr, uint32_t* sd_end, uint64_t* s_scan,
+                                                   uint32_t* ns) {
+    const uint32_t per = (n + THREADS - 1) / THREADS;
+    const uint32_t b = threadIdx.x * per, e = min(b + per, n);
+    uint64_t acc = 0;  // (non-empty count << 32) | product count
+    for (uint32_t i = b; i < e; ++i) {
+        uint32_t len;
+        get_seg(s, r, s0 + i, len);
+        if (len) acc += (1ull << 32) + len;
+    }
+    uint64_t tot;
+    const uint64_t ex = block_exclusive_scan<uint64_t>(acc, s_scan, &tot);
+    uint32_t k = uint32_t(ex >> 32), run = uint32_t(ex);
+    for (uint32_t i = b; i < e; ++i) {
+        uint32_t len;
+        const idx_t* p = get_seg(s, r, s0 + i, len);
+        if (len) {
+            sd_ptr[k] = p - run;
+            run += len;
+            sd_end[k] = run;
+            ++k;
+        }
+    }
+    __syncthreads();
+    *ns = uint32_t(tot >> 32);
+    return uint32_t(tot);
+}
+
+// Call f(c) for every product of row r.  Warps take chunks of 32*U
+// consecutive products; per 32-product step a lane loads one candidate
+// segment (32 consecutive segments cover 32 consecutive products), a 5-step
+// shuffle search finds each lane's segment, and the U loads of a chunk
+// are issued before any insert.  Ends with a barrier.
+template <int THREADS, int U, typename F>
+__device__ __forceinline__ void block_products(const SegSource& s, idx_t r, const idx_t** sd_ptr,
+                                               uint32_t* sd_end, uint32_t batch, uint64_t* s_scan, F&& f) {
+    constexpr uint32_t NW = THREADS / 32, CH = 32 * U;
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t nseg = num_segs(s, r);
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
-        const uint32_t n = min(batch, nseg - s0);
-        const uint32_t per = (n + THREADS - 1) / THREADS;
-        const uint32_t b = threadIdx.x * per, e = min(b + per, n);
-        uint64_t sum = 0;
-        for (uint32_t i = b; i < e; ++i) {
-            uint32_t len;
-            sd_ptr[i] = get_seg(s, r, s0 + i, len);
-            sd_end[i] = len;  // temporarily the length
-            sum += len;
-        }
-        uint64_t tot;
-        uint64_t run = block_exclusive_scan<uint64_t>(sum, s_scan, &tot);
-        for (uint32_t i = b; i < e; ++i) {
-            run += sd_end[i];
-            sd_end[i] = uint32_t(run);
-        }
-        __syncthreads();
-        const uint32_t total = uint32_t(tot);
-        for (uint32_t q0 = threadIdx.x; q0 < total; q0 += THREADS * kFlatUnroll) {
-            idx_t v[kFlatUnroll];
+        uint32_t ns;
+        const uint32_t total = stage_segments<THREADS>(s, r, s0, min(batch, nseg - s0), sd_ptr, sd_end, s_scan, &ns);
+        for (uint32_t base = wib * CH; base < total; base += NW * CH) {
+            uint32_t lo = 0, hi = ns - 1;  // segment holding product `base`
+            while (lo < hi) {
+                const uint32_t mid = (lo + hi) >> 1;
+                if (sd_end[mid] <= base) lo = mid + 1; else hi = mid;
+            }
+            uint32_t sb = lo;
+            idx_t v[U];
 #pragma unroll
-            for (int u = 0; u < kFlatUnroll; ++u) {
-                const uint32_t q = q0 + u * THREADS;
-                v[u] = kEmpty;
-                if (q < total) {
-                    uint32_t lo = 0, hi = n - 1;  // first segment whose end > q
-                    while (lo < hi) {
-                        const uint32_t mid = (lo + hi) >> 1;
-                        if (sd_end[mid] <= q) lo = mid + 1; else hi = mid;
-                    }
-                    const uint32_t st = lo ? sd_end[lo - 1] : 0u;
-                    v[u] = __ldg(sd_ptr[lo] + (q - st));
+            for (int u = 0; u < U; ++u) {
+                const uint32_t qb = base + 32u * u, q = qb + lane;
+                const uint32_t cand = sb + lane;
+                const uint32_t E = cand < ns ? sd_end[cand] : 0xFFFFFFFFu;
+                const unsigned long long P = cand < ns ? (unsigned long long)sd_ptr[cand] : 0ull;
+                uint32_t pos = 0;
+#pragma unroll
+                for (int st = 16; st > 0; st >>= 1) {
+                    const uint32_t t = __shfl_sync(FULL, E, pos + st - 1);
+                    if (t <= q) pos += st;
                 }
+                const idx_t* ps = (const idx_t*)__shfl_sync(FULL, P, pos > 31 ? 31 : pos);
+                v[u] = q < total ? __ldg(ps + q) : kEmpty;
+                sb += __popc(__ballot_sync(FULL, E <= qb + 32));
             }
 #pragma unroll
-            for (int u = 0; u < kFlatUnroll; ++u)
+            for (int u = 0; u < U; ++u)
                 if (v[u] != kEmpty) f(v[u]);
         }
-        __syncthreads();  // smem descriptors are reused by the next batch
+        __syncthreads();  // descriptors are reused by the next batch
     }
 }
 
-// Ordered, coalesced emission of the set bits of bm[0..nwords) as columns
-// base_col + 32*i + b.  Warp w owns a contiguous run of words; one block scan
-// of the per-warp counts.  Returns the count (all threads).
+// Block scan of per-warp counts held in s_w[0..NW); s_w[w] becomes the
+// warp's output base, s_w[32] the total.
+template <int NW>
+__device__ __forceinline__ void scan_warp_counts(uint32_t* s_w) {
+    const unsigned lane = lane_id();
+    if ((threadIdx.x >> 5) == 0) {
+        const uint32_t v = lane < NW ? s_w[lane] : 0u;
+        const uint32_t inc = warp_inclusive_scan(v);
+        if (lane < NW) s_w[lane] = inc - v;
+        if (lane == NW - 1) s_w[32] = inc;
+    }
+    __syncthreads();
+}
+
+// Ordered emission of the set bits of bm[0..nwords) as base_col + 32 i + b,
+// warp w owning words [w*chunk, (w+1)*chunk).  Returns the count.
+template <int NW>
 __device__ __forceinline__ uint32_t emit_bitmap(const uint32_t* bm, uint32_t nwords, uint64_t base_col,
                                                 idx_t* __restrict__ out, uint32_t* s_w) {
-    const unsigned lane = lane_id(), wib = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const uint32_t chunk = ((nwords + nw - 1) / nw + 31) & ~31u;
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
+    const uint32_t chunk = ((nwords + NW - 1) / NW + 31) & ~31u;
     const uint32_t b = wib * chunk, e = min(b + chunk, nwords);
     uint32_t cnt = 0;
     for (uint32_t i = b + lane; i < e; i += 32) cnt += __popc(bm[i]);
     cnt = warp_sum(cnt);
     if (lane == 0) s_w[wib] = cnt;
     __syncthreads();
-    if (wib == 0) {
-        uint32_t v = lane < nw ? s_w[lane] : 0u;
-        uint32_t inc = warp_inclusive_scan(v);
-        if (lane < nw) s_w[lane] = inc - v;
-        if (lane == nw - 1) s_w[32] = inc;
-    }
-    __syncthreads();
+    scan_warp_counts<NW>(s_w);
     uint32_t pos = s_w[wib];
     for (uint32_t i0 = b; i0 < e; i0 += 32) {
         const uint32_t i = i0 + lane;
@@ -217,14 +252,14 @@ __device__ __forceinline__ uint32_t emit_bitmap(const uint32_t* bm, uint32_t nwo
     return total;
 }
 
-// Ordered, coalesced emission of an order-preserving hash table: clusters
-// (maximal runs of occupied slots) are ordered relative to each other, so an
-// element at slot i goes to  (#occupied slots before its cluster start cs)
-// + (its rank inside the cluster)  — no in-smem sort, no extra barrier.
+// Ordered emission of an order-preserving hash table: clusters (maximal runs
+// of occupied slots) are mutually ordered, so the element at slot i goes to
+// (#occupied slots before its cluster start cs) + (its rank in the cluster).
+template <int NW>
 __device__ __forceinline__ uint32_t emit_table_ranked(const idx_t* tab, uint32_t nslots, idx_t* __restrict__ out,
                                                       uint32_t* s_w) {
-    const unsigned lane = lane_id(), wib = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const uint32_t chunk = ((nslots + nw - 1) / nw + 31) & ~31u;
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
+    const uint32_t chunk = ((nslots + NW - 1) / NW + 31) & ~31u;
     const uint32_t b = wib * chunk, e = min(b + chunk, nslots);
     uint32_t cnt = 0;
     for (uint32_t i0 = b; i0 < e; i0 += 32) {
@@ -233,13 +268,7 @@ __device__ __forceinline__ uint32_t emit_table_ranked(const idx_t* tab, uint32_t
     }
     if (lane == 0) s_w[wib] = cnt;
     __syncthreads();
-    if (wib == 0) {
-        uint32_t v = lane < nw ? s_w[lane] : 0u;
-        uint32_t inc = warp_inclusive_scan(v);
-        if (lane < nw) s_w[lane] = inc - v;
-        if (lane == nw - 1) s_w[32] = inc;
-    }
-    __syncthreads();
+    scan_warp_counts<NW>(s_w);
     uint32_t pos = s_w[wib];
     const uint32_t lt = (1u << lane) - 1u;
     for (uint32_t i0 = b; i0 < e; i0 += 32) {
@@ -262,6 +291,281 @@ __device__ __forceinline__ uint32_t emit_table_ranked(const idx_t* tab, uint32_t
     const uint32_t total = s_w[32];
     __syncthreads();
     return total;
+}
+
+__device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, int threads) {
+    // p is 16-byte aligned; vector stores for the bulk
+    uint4* p4 = reinterpret_cast<uint4*>(p);
+    const uint4 v4 = make_uint4(v, v, v, v);
+    for (uint32_t i = threadIdx.x; i < n / 4; i += threads) p4[i] = v4;
+    for (uint32_t i = (n & ~3u) + threadIdx.x; i < n; i += threads) p[i] = v;
+}
+
+// ---- 4b. block hash / span-bitmap bins --------------------------------------
+// Bucketed ORDER-PRESERVING hash: bucket b = floor((c - lo) * nb / span) is
+// monotone in c, so buckets are mutually ordered; each bucket has 8 slots
+// (mean load 4), claimed by atomicCAS scanning from slot 0 (the scan order
+// makes duplicates meet).  A full bucket spills to a small monotone
+// linear-probing overflow table.  Emission: per-thread runs of buckets, a
+// block scan of their counts, an 8-input Batcher network sorts each bucket
+// in registers, and the (few) overflow elements are merged by rank:
+//   main v at bucket b, index j : prefix(b) + j + #(overflow < v)
+//   overflow x (i-th smallest)  : prefix(b_x) + #(bucket b_x < x) + i
+__device__ __forceinline__ void cswap(idx_t& a, idx_t& b) {
+    const idx_t x = min(a, b), y = max(a, b);
+    a = x;
+    b = y;
+}
+__device__ __forceinline__ void sort8(idx_t (&v)[8]) {  // Batcher odd-even merge sort, 19 comparators
+    cswap(v[0], v[1]); cswap(v[2], v[3]); cswap(v[4], v[5]); cswap(v[6], v[7]);
+    cswap(v[0], v[2]); cswap(v[1], v[3]); cswap(v[4], v[6]); cswap(v[5], v[7]);
+    cswap(v[1], v[2]); cswap(v[5], v[6]);
+    cswap(v[0], v[4]); cswap(v[1], v[5]); cswap(v[2], v[6]); cswap(v[3], v[7]);
+    cswap(v[2], v[4]); cswap(v[3], v[5]);
+    cswap(v[1], v[2]); cswap(v[3], v[4]); cswap(v[5], v[6]);
+}
+__device__ __forceinline__ uint32_t lower_bound_smem(const idx_t* a, uint32_t n, idx_t key) {
+    uint32_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (a[mid] < key) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+constexpr uint32_t kOvSlack = 128;
+
+// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] | ovt[OVS+kOvSlack] | ovs[OVS]
+template <int THREADS, uint32_t MAXB, uint32_t OVS, uint32_t BATCH, int MINB, int FLATU>
+__global__ void __launch_bounds__(THREADS, MINB)
+hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
+                const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
+                idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
+                uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
+    constexpr int NW = THREADS / 32;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
+    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
+    idx_t* tab = reinterpret_cast<idx_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
+    idx_t* ovt = tab + MAXB * 8;
+    idx_t* ovs = ovt + OVS + kOvSlack;
+    __shared__ uint64_t s_scan[33];
+    __shared__ uint32_t s_w[33];
+    __shared__ uint32_t s_base[THREADS];
+    __shared__ uint32_t s_item, s_flag, s_novf;
+    const uint32_t lo_i = bounds[0], hi_i = bounds[1];
+    for (;;) {
+        if (threadIdx.x == 0) {
+            s_item = lo_i + atomicAdd(work, 1u);
+            s_flag = 0;
+            s_novf = 0;
+        }
+        __syncthreads();
+        const uint32_t item = s_item;
+        if (item >= hi_i) break;
+        const idx_t r = rows[item];
+        const uint32_t u = uint32_t(ub[r]);
+        uint32_t clo = 0, chi = ncols - 1;
+        if (range) {
+            const uint2 rg = range[r];
+            clo = rg.x;
+            chi = rg.y;
+        }
+        const uint64_t span = uint64_t(chi) - clo + 1;
+        const uint32_t nb = min(max((u + 3) / 4, 1u), MAXB);
+        const uint64_t words = (span + 31) >> 5;
+        idx_t* out = scratch + soff[r];
+        if (words <= 8ull * nb) {  // the span bitmap is no larger than the table
+            const uint32_t nw = uint32_t(words);
+            fill_words(tab, nw, 0u, THREADS);
+            __syncthreads();
+            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+                const uint32_t d = c - clo;
+                atomicOr(&tab[d >> 5], 1u << (d & 31));
+            });
+            const uint32_t n = emit_bitmap<NW>(tab, nw, clo, out, s_w);
+            if (threadIdx.x == 0) counts[r] = n;
+            continue;  // emit_bitmap ends with a barrier
+        }
+        const uint32_t ovn = min(max(u / 16, 64u), OVS);
+        const uint32_t ovslots = ovn + kOvSlack;
+        fill_words(tab, nb * 8, kEmpty, THREADS);
+        fill_words(ovt, ovslots, kEmpty, THREADS);
+        __syncthreads();
+        const uint64_t bscale = (uint64_t(nb) << 32) / span;
+        const uint64_t oscale = (uint64_t(ovn) << 32) / span;
+        block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+            const uint64_t d = uint64_t(c - clo);
+            idx_t* bk = tab + uint32_t((d * bscale) >> 32) * 8;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const idx_t cur = bk[k];
+                if (cur == c) return;
+                if (cur == kEmpty) {
+                    const idx_t old = atomicCAS(&bk[k], kEmpty, c);
+                    if (old == kEmpty || old == c) return;
+                }
+            }
+            // bucket full: overflow table (monotone linear probing, no wrap)
+            uint32_t h = uint32_t((d * oscale) >> 32);
+            for (uint32_t probe = 0;; ++probe) {
+                const idx_t cur = ovt[h];
+                if (cur == c) return;
+                if (cur == kEmpty) {
+                    const idx_t old = atomicCAS(&ovt[h], kEmpty, c);
+                    if (old == kEmpty) {
+                        atomicAdd(&s_novf, 1u);
+                        return;
+                    }
+                    if (old == c) return;
+                }
+                if (++h >= ovslots || probe >= kMaxProbe) {
+                    s_flag = 1;  // hand the row to the bitmap bin
+                    return;
+                }
+            }
+        });
+        if (s_flag) {
+            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            __syncthreads();  // everyone has read s_flag / s_item before reuse
+            continue;
+        }
+        const uint32_t novf = s_novf;
+        if (novf) emit_table_ranked<NW>(ovt, ovslots, ovs, s_w);  // sorted overflow -> ovs (smem)
+        // main buckets: thread t owns buckets [t*k, (t+1)*k)
+        const uint32_t k = (nb + THREADS - 1) / THREADS;
+        const uint32_t b0 = threadIdx.x * k, b1 = min(b0 + k, nb);
+        uint64_t cnt = 0;
+        for (uint32_t b = b0; b < b1; ++b) {
+            const uint4* p4 = reinterpret_cast<const uint4*>(tab + b * 8);
+            const uint4 x = p4[0], y = p4[1];
+            cnt += (x.x != kEmpty) + (x.y != kEmpty) + (x.z != kEmpty) + (x.w != kEmpty) +
+                   (y.x != kEmpty) + (y.y != kEmpty) + (y.z != kEmpty) + (y.w != kEmpty);
+        }
+        uint64_t total_main;
+        uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(cnt, s_scan, &total_main));
+        s_base[threadIdx.x] = pos;
+        for (uint32_t b = b0; b < b1; ++b) {
+            const uint4* p4 = reinterpret_cast<const uint4*>(tab + b * 8);
+            const uint4 x = p4[0], y = p4[1];
+            idx_t v[8] = {x.x, x.y, x.z, x.w, y.x, y.y, y.z, y.w};
+            sort8(v);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                if (v[j] != kEmpty) {
+                    const uint32_t extra = novf ? lower_bound_smem(ovs, novf, v[j]) : 0u;
+                    out[pos + extra] = v[j];
+                    ++pos;
+                }
+            }
+        }
+        if (novf) {
+            __syncthreads();  // s_base complete
+            for (uint32_t i = threadIdx.x; i < novf; i += THREADS) {
+                const idx_t xv = ovs[i];
+                const uint32_t b = uint32_t((uint64_t(xv - clo) * bscale) >> 32);
+                const uint32_t owner = b / k;
+                uint32_t p = s_base[owner];
+                for (uint32_t bb = owner * k; bb <= b; ++bb)
+                    for (int j = 0; j < 8; ++j) {
+                        const idx_t w = tab[bb * 8 + j];
+                        p += (w != kEmpty) && (bb < b || w < xv);
+                    }
+                out[p + i] = xv;
+            }
+        }
+        if (threadIdx.x == 0) counts[r] = uint32_t(total_main) + novf;
+        __syncthreads();
+    }
+}
+
+// ---- 4c. block two-level bitmap bin ------------------------------------------
+// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | bm[kDenseBits/32] | top[kDenseBits/1024]
+// top bit t set <=> bm word t may be non-zero.  Emission walks the top level,
+// so clearing and emitting cost O(words touched + kDenseBits/1024).
+template <int THREADS, uint32_t BATCH, int FLATU>
+__global__ void __launch_bounds__(THREADS)
+dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
+                 const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
+                 const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts, uint32_t* __restrict__ work) {
+    constexpr int NW = THREADS / 32;
+    constexpr uint32_t kWords = kDenseBits / 32, kTop = kWords / 32;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
+    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
+    uint32_t* bm = reinterpret_cast<uint32_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
+    uint32_t* top = bm + kWords;
+    __shared__ uint64_t s_scan[33];
+    __shared__ uint32_t s_w[33];
+    __shared__ uint32_t s_item;
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
+    fill_words(bm, kWords + kTop, 0u, THREADS);  // kept clean between rows
+    __syncthreads();
+    for (;;) {
+        if (threadIdx.x == 0) s_item = bounds[0] + atomicAdd(work, 1u);
+        __syncthreads();
+        const uint32_t item = s_item;
+        if (item >= bounds[1]) break;
+        const idx_t r = rows[item];
+        uint32_t clo = 0, chi = ncols - 1;
+        if (range) {
+            const uint2 rg = range[r];
+            clo = rg.x;
+            chi = rg.y;
+        }
+        const uint64_t span = uint64_t(chi) - clo + 1;
+        const uint32_t nwin = uint32_t((span + kDenseBits - 1) / kDenseBits);
+        idx_t* out = scratch + soff[r];
+        uint32_t written = 0;
+        for (uint32_t w = 0; w < nwin; ++w) {
+            const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseBits;
+            const uint64_t whi = min(wlo + kDenseBits, uint64_t(chi) + 1);
+            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+                if (c >= wlo && c < whi) {
+                    const uint32_t d = uint32_t(c - wlo);
+                    const uint32_t bit = 1u << (d & 31);
+                    const uint32_t old = atomicOr(&bm[d >> 5], bit);
+                    if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
+                }
+            });
+            // emission over the top level: warp w owns top words [w*tc, (w+1)*tc)
+            constexpr uint32_t tc = kTop / NW;
+            const uint32_t tb = wib * tc;
+            uint32_t cnt = 0;
+            for (uint32_t t = tb; t < tb + tc; ++t) {  // warp-uniform loop over top words
+                const uint32_t tw = top[t];
+                if (tw == 0) continue;
+                const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                cnt += __popc(word);
+            }
+            cnt = warp_sum(cnt);
+            if (lane == 0) s_w[wib] = cnt;
+            __syncthreads();
+            scan_warp_counts<NW>(s_w);
+            uint32_t pos = s_w[wib];
+            for (uint32_t t = tb; t < tb + tc; ++t) {
+                const uint32_t tw = top[t];
+                if (tw == 0) continue;
+                uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                if ((tw >> lane) & 1u) bm[t * 32 + lane] = 0u;  // clean for the next row/window
+                const uint32_t c = __popc(word);
+                const uint32_t inc = warp_inclusive_scan(c);
+                uint32_t o = pos + inc - c;
+                const uint64_t colbase = wlo + (uint64_t(t * 32 + lane) << 5);
+                while (word) {
+                    const int bit = __ffs(word) - 1;
+                    word &= word - 1;
+                    out[written + o++] = idx_t(colbase + bit);
+                }
+                pos += __shfl_sync(FULL, inc, 31);
+                __syncwarp();
+                if (lane == 0) top[t] = 0u;
+            }
+            written += s_w[32];
+            __syncthreads();
+        }
+        if (threadIdx.x == 0) counts[r] = written;
+    }
 }
 
 // ---- 1. binning ------------------------------------------------------------
@@ -406,135 +710,6 @@ warp_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     }
 }
 
-// ---- 4b. block hash / small-span bitmap bins -------------------------------
-__device__ __forceinline__ uint32_t next_pow2(uint32_t v) {
-    return v <= 1 ? 1u : 1u << (32 - __clz(v - 1));
-}
-
-// dynamic smem: table[TMAX + kSlack] | sd_ptr[BATCH] | sd_end[BATCH]
-template <int THREADS, uint32_t TMAX, uint32_t BATCH>
-__global__ void __launch_bounds__(THREADS)
-hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
-                const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
-                idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
-                uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
-    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
-    idx_t* tab = reinterpret_cast<idx_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
-    __shared__ uint64_t s_scan[33];
-    __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_item, s_flag;
-    const uint32_t lo_i = bounds[0], hi_i = bounds[1];
-    for (;;) {
-        if (threadIdx.x == 0) {
-            s_item = lo_i + atomicAdd(work, 1u);
-            s_flag = 0;
-        }
-        __syncthreads();
-        const uint32_t item = s_item;
-        if (item >= hi_i) break;
-        const idx_t r = rows[item];
-        const uint32_t u = uint32_t(ub[r]);
-        uint32_t clo = 0, chi = ncols - 1;
-        if (range) {
-            uint2 rg = range[r];
-            clo = rg.x;
-            chi = rg.y;
-        }
-        const uint64_t span = uint64_t(chi) - clo + 1;
-        const uint32_t T = min(next_pow2(2 * u), TMAX);
-        const uint64_t words = (span + 31) >> 5;
-        const bool bitmap = words <= T;
-        const uint32_t nslots = bitmap ? uint32_t(words) : T + kSlack;
-        const idx_t fill = bitmap ? 0u : kEmpty;
-        for (uint32_t i = threadIdx.x; i < nslots; i += THREADS) tab[i] = fill;
-        __syncthreads();
-        if (bitmap) {
-            block_flat<THREADS>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
-                const uint32_t d = c - clo;
-                atomicOr(&tab[d >> 5], 1u << (d & 31));
-            });
-            const uint32_t n = emit_bitmap(tab, nslots, clo, scratch + soff[r], s_w);
-            if (threadIdx.x == 0) counts[r] = n;
-            continue;  // emit_bitmap ends with a barrier
-        }
-        // order-preserving home slot: floor((c - clo) * T / span) via a
-        // 32.32 fixed-point scale; monotone in c and < T
-        const uint64_t scale = (uint64_t(T) << 32) / span;
-        block_flat<THREADS>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
-            uint32_t h = uint32_t((uint64_t(c - clo) * scale) >> 32);
-            for (uint32_t probe = 0;; ++probe) {
-                const idx_t cur = tab[h];
-                if (cur == c) break;
-                if (cur == kEmpty) {
-                    const idx_t old = atomicCAS(&tab[h], kEmpty, c);
-                    if (old == kEmpty || old == c) break;
-                }
-                if (++h >= nslots || probe >= kMaxProbe) {
-                    s_flag = 1;  // long cluster: hand the row to the bitmap bin
-                    break;
-                }
-            }
-        });
-        // block_flat ends with a barrier
-        if (s_flag) {
-            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
-            __syncthreads();  // everyone has read s_flag / s_item before reuse
-            continue;
-        }
-        const uint32_t n = emit_table_ranked(tab, nslots, scratch + soff[r], s_w);
-        if (threadIdx.x == 0) counts[r] = n;
-    }
-}
-
-// ---- 4c. block bitmap bin ----------------------------------------------------
-// dynamic smem: bitmap[kDenseMaxBits/32] | sd_ptr[kDenseBatch] | sd_end[kDenseBatch]
-__global__ void __launch_bounds__(kDenseThreads)
-dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
-                 const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
-                 const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts, uint32_t* __restrict__ work) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
-    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + kDenseBatch * sizeof(void*));
-    uint32_t* bm = reinterpret_cast<uint32_t*>(smem_raw + kDenseBatch * (sizeof(void*) + sizeof(uint32_t)));
-    __shared__ uint64_t s_scan[33];
-    __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_item;
-    for (;;) {
-        if (threadIdx.x == 0) s_item = bounds[0] + atomicAdd(work, 1u);
-        __syncthreads();
-        const uint32_t item = s_item;
-        if (item >= bounds[1]) break;
-        const idx_t r = rows[item];
-        uint32_t clo = 0, chi = ncols - 1;
-        if (range) {
-            uint2 rg = range[r];
-            clo = rg.x;
-            chi = rg.y;
-        }
-        const uint64_t span = uint64_t(chi) - clo + 1;
-        const uint32_t nwin = uint32_t((span + kDenseMaxBits - 1) / kDenseMaxBits);
-        idx_t* out = scratch + soff[r];
-        uint32_t written = 0;
-        for (uint32_t w = 0; w < nwin; ++w) {
-            const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseMaxBits;
-            const uint64_t whi = min(wlo + kDenseMaxBits, uint64_t(chi) + 1);
-            const uint32_t nwords = uint32_t((whi - wlo + 31) >> 5);
-            for (uint32_t i = threadIdx.x; i < nwords; i += blockDim.x) bm[i] = 0;
-            __syncthreads();
-            block_flat<kDenseThreads>(src, r, sd_ptr, sd_end, kDenseBatch, s_scan, [&](idx_t c) {
-                if (c >= wlo && c < whi) {
-                    const uint32_t d = uint32_t(c - wlo);
-                    atomicOr(&bm[d >> 5], 1u << (d & 31));
-                }
-            });
-            written += emit_bitmap(bm, nwords, wlo, out + written, s_w);
-        }
-        if (threadIdx.x == 0) counts[r] = written;
-    }
-}
-
 // ---- 6. compaction -------------------------------------------------------------
 __global__ void compact_kernel(const idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff,
                                const uint64_t* __restrict__ rowptr, idx_t nrows,
@@ -552,31 +727,32 @@ __global__ void compact_kernel(const idx_t* __restrict__ scratch, const uint64_t
 }  // namespace
 
 // ------------------------------------------------------------------------------
-struct AuxStreams {
-    cudaStream_t s[3] = {nullptr, nullptr, nullptr};
-    cudaEvent_t fork = nullptr, join[3] = {nullptr, nullptr, nullptr};
-    int device = -1;
-};
-static AuxStreams g_aux;
-
 constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
-constexpr size_t kHashSSmem = (2 * kHashSMaxUb + kSlack) * sizeof(idx_t) + kHashSBatch * kSegBytes;
-constexpr size_t kHashLSmem = (2 * kHashLMaxUb + kSlack) * sizeof(idx_t) + kHashLBatch * kSegBytes;
-constexpr size_t kDenseSmem = kDenseMaxBits / 8 + kDenseBatch * kSegBytes;
-#define HASH_S hash_bin_kernel<kHashSThreads, 2 * kHashSMaxUb, kHashSBatch>
-#define HASH_L hash_bin_kernel<kHashLThreads, 2 * kHashLMaxUb, kHashLBatch>
+constexpr uint32_t kSBatch = 512, kLBatch = 384, kXBatch = 256, kDBatch = 2048;
+constexpr uint32_t kSBuckets = kHashSMaxUb / 4, kLBuckets = kHashLMaxUb / 4, kXBuckets = kHashXMaxUb / 4;
+constexpr uint32_t kSOvs = 128, kLOvs = 384, kXOvs = 1536;
+constexpr size_t hash_smem(uint32_t batch, uint32_t buckets, uint32_t ovs) {
+    return batch * kSegBytes + (buckets * 8 + ovs + kOvSlack + ovs) * sizeof(idx_t);
+}
+constexpr size_t kSSmem = hash_smem(kSBatch, kSBuckets, kSOvs);
+constexpr size_t kLSmem = hash_smem(kLBatch, kLBuckets, kLOvs);
+constexpr size_t kXSmem = hash_smem(kXBatch, kXBuckets, kXOvs);
+constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
+#define HASH_S hash_bin_kernel<256, kSBuckets, kSOvs, kSBatch, 6, 4>
+#define HASH_L hash_bin_kernel<512, kLBuckets, kLOvs, kLBatch, 3, 4>
+#define HASH_X hash_bin_kernel<1024, kXBuckets, kXOvs, kXBatch, 1, 8>
+#define DENSE dense_bin_kernel<1024, kDBatch, 8>
+static_assert(kLSmem + 2 * 1024 + 700 <= 227 * 1024 / 3, "hash-L: 3 blocks per SM");
+static_assert(kXSmem + 4 * 1024 + 700 <= 227 * 1024, "hash-X fits");
 
-static void ensure_aux() {
-    if (g_aux.device == ctx().device) return;
-    for (int i = 0; i < 3; ++i) {
-        CUDA_CHECK(cudaStreamCreateWithFlags(&g_aux.s[i], cudaStreamNonBlocking));
-        CUDA_CHECK(cudaEventCreateWithFlags(&g_aux.join[i], cudaEventDisableTiming));
-    }
-    CUDA_CHECK(cudaEventCreateWithFlags(&g_aux.fork, cudaEventDisableTiming));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH_S, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kHashSSmem)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH_L, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kHashLSmem)));
-    CUDA_CHECK(cudaFuncSetAttribute(dense_bin_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDenseSmem)));
-    g_aux.device = ctx().device;
+static void ensure_attrs() {
+    static int done_dev = -1;
+    if (done_dev == ctx().device) return;
+    CUDA_CHECK(cudaFuncSetAttribute(HASH_S, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kSSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH_L, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kLSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH_X, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kXSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(DENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDSmem)));
+    done_dev = ctx().device;
 }
 
 void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, const uint2* range,
@@ -587,19 +763,19 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
         matrix_set_empty(out);
         return;
     }
-    ensure_aux();
-    // 1. bins
+    ensure_attrs();
+    // 1-3. bins
     DevBuf<uint64_t> cap(size_t(nrows) + 1);
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    // meta: hist[9] binoff[10] cursor[9] work[4] ovf[2]
+    // meta: hist[10] binoff[11] cursor[10] work[6] ovf[2]
     DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
     uint32_t* binoff = meta.p + 10;
     uint32_t* cursor = meta.p + 21;
     uint32_t* work = meta.p + 31;
-    uint32_t* ovf = meta.p + 36;  // ovf[0] = 0 (list start), ovf[1] = count
+    uint32_t* ovf = meta.p + 38;  // ovf[0] = 0 (list start), ovf[1] = count
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
     const unsigned gb = (unsigned)std::min<uint64_t>(ceil_div(nrows, 256), uint64_t(nsm) * 8);
     bin_count_kernel<<<gb, 256, 0, st>>>(ub, nrows, ncols, cap.p, bin.p, counts.p, hist);
@@ -620,41 +796,40 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<idx_t> scratch(scratch_total);
     DevBuf<idx_t> ovf_rows(nrows);
 
-    // 4. per-bin kernels on forked streams
-    CUDA_CHECK(cudaEventRecord(g_aux.fork, st));
-    for (int i = 0; i < 3; ++i) CUDA_CHECK(cudaStreamWaitEvent(g_aux.s[i], g_aux.fork, 0));
+    // 4. per-bin kernels, heaviest first, back to back on the library stream
+    //    (persistent grids sized to the SM count x residency; rows are handed
+    //    out by an atomic work counter, so heavy rows balance dynamically)
+    int t;
+    t = ktime_begin("dense", st);
+    DENSE<<<nsm, 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols, scratch.p, soff.p,
+                                     counts.p, work);
+    ktime_end(t);
+    t = ktime_begin("hash_x", st);
+    HASH_X<<<nsm, 1024, kXSmem, st>>>(src, rows.p, binoff + BIN_HASH_X, ub, range, ncols, scratch.p, soff.p,
+                                      counts.p, work + 1, ovf_rows.p, ovf);
+    ktime_end(t);
+    t = ktime_begin("hash_l", st);
+    HASH_L<<<nsm * 3, 512, kLSmem, st>>>(src, rows.p, binoff + BIN_HASH_L, ub, range, ncols, scratch.p, soff.p,
+                                         counts.p, work + 2, ovf_rows.p, ovf);
+    ktime_end(t);
+    t = ktime_begin("hash_s", st);
+    HASH_S<<<nsm * 6, 256, kSSmem, st>>>(src, rows.p, binoff + BIN_HASH_S, ub, range, ncols, scratch.p, soff.p,
+                                         counts.p, work + 3, ovf_rows.p, ovf);
+    ktime_end(t);
+    // rows whose hash probes ran long: bitmap path
+    DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 4);
+    count_launch(5);
+    check_launch("block bins");
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
-    {
-        cudaStream_t s3 = g_aux.s[2];  // heaviest first
-        dense_bin_kernel<<<nsm, kDenseThreads, kDenseSmem, s3>>>(
-            src, rows.p, binoff + BIN_DENSE, range, ncols, scratch.p, soff.p, counts.p, work);
-        count_launch();
-        check_launch("dense_bin_kernel");
-        cudaStream_t s2 = g_aux.s[1];
-        HASH_L<<<nsm * 3, kHashLThreads, kHashLSmem, s2>>>(
-            src, rows.p, binoff + BIN_HASH_L, ub, range, ncols, scratch.p, soff.p, counts.p, work + 1,
-            ovf_rows.p, ovf);
-        HASH_S<<<nsm * 7, kHashSThreads, kHashSSmem, s2>>>(
-            src, rows.p, binoff + BIN_HASH_S, ub, range, ncols, scratch.p, soff.p, counts.p, work + 2,
-            ovf_rows.p, ovf);
-        // rows whose hash probes ran long: bitmap path
-        dense_bin_kernel<<<nsm, kDenseThreads, kDenseSmem, s2>>>(
-            src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 3);
-        count_launch(3);
-        check_launch("hash_bin_kernel");
-        cudaStream_t s1 = g_aux.s[0];
-        warp_bin_kernel<16><<<gw, 256, 0, s1>>>(src, rows.p, binoff, BIN_W16, scratch.p, soff.p, counts.p);
-        warp_bin_kernel<8><<<gw, 256, 0, s1>>>(src, rows.p, binoff, BIN_W8, scratch.p, soff.p, counts.p);
-        warp_bin_kernel<4><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W4, scratch.p, soff.p, counts.p);
-        warp_bin_kernel<2><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W2, scratch.p, soff.p, counts.p);
-        warp_bin_kernel<1><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W1, scratch.p, soff.p, counts.p);
-        count_launch(5);
-        check_launch("warp_bin_kernel");
-    }
-    for (int i = 0; i < 3; ++i) {
-        CUDA_CHECK(cudaEventRecord(g_aux.join[i], g_aux.s[i]));
-        CUDA_CHECK(cudaStreamWaitEvent(st, g_aux.join[i], 0));
-    }
+    t = ktime_begin("warp_bins", st);
+    warp_bin_kernel<16><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W16, scratch.p, soff.p, counts.p);
+    warp_bin_kernel<8><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W8, scratch.p, soff.p, counts.p);
+    warp_bin_kernel<4><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W4, scratch.p, soff.p, counts.p);
+    warp_bin_kernel<2><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W2, scratch.p, soff.p, counts.p);
+    warp_bin_kernel<1><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W1, scratch.p, soff.p, counts.p);
+    ktime_end(t);
+    count_launch(5);
+    check_launch("warp_bin_kernel");
     // 5. row offsets
     DevBuf<off_t64> rowptr(size_t(nrows) + 1);
     exclusive_scan_u32(counts.p, rowptr.p, nrows);
@@ -663,12 +838,22 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<idx_t> colidx(nnz);
     if (nnz) {
         const unsigned gc = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(nrows) * 32, 256), uint64_t(nsm) * 16);
+        t = ktime_begin("compact", st);
         compact_kernel<<<gc, 256, 0, st>>>(scratch.p, soff.p, rowptr.p, nrows, colidx.p);
+        ktime_end(t);
         count_launch();
         check_launch("compact_kernel");
     }
     size_t rcap = rowptr.n, ccap = colidx.n;
     matrix_replace(out, rowptr.detach(), rcap, colidx.detach(), ccap, nnz);
+}
+
+void engine_thresholds(uint64_t* out, uint32_t* n) {
+    // ub upper limits of bins W1, W2, W4, W8, W16, HASH_S, HASH_L, HASH_X (DENSE above)
+    const uint64_t t[8] = {32, 64, 128, 256, kWarpMaxUb, kHashSMaxUb, kHashLMaxUb, kHashXMaxUb};
+    const uint32_t k = *n < 8 ? *n : 8;
+    for (uint32_t i = 0; i < k; ++i) out[i] = t[i];
+    *n = 8;
 }
 
 }  // namespace spbla

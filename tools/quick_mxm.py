@@ -20,6 +20,13 @@ rp, ci = A.device_tensors()
 lens = rp[1:] - rp[:-1]
 prods = int(lens[ci.long()].sum())
 print("products", prods, flush=True)
+rows_of = torch.repeat_interleave(torch.arange(n, device="cuda"), lens)
+ub = torch.zeros(n, dtype=torch.int64, device="cuda").index_add_(0, rows_of, lens[ci.long()])
+edges = [0, 1, 33, 65, 129, 257, 513, 2049, 8193, 1 << 62]
+for lo, hi in zip(edges[:-1], edges[1:]):
+    m = (ub >= lo) & (ub < hi)
+    print(f"ub [{lo},{hi}) rows {int(m.sum()):9d} products {int(ub[m].sum())/prods*100:6.2f}%", flush=True)
+del rows_of
 st = torch.cuda.current_stream()
 for i in range(int(os.environ.get("ITERS", "5"))):
     e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
