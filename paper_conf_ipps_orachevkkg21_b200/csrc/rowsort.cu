@@ -45,8 +45,8 @@ enum {
 };
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 512
 constexpr uint64_t kHashSMaxUb = 2048;
-constexpr uint64_t kHashLMaxUb = 8192;
-constexpr uint64_t kHashXMaxUb = 24576;
+constexpr uint64_t kHashLMaxUb = 6144;
+constexpr uint64_t kHashXMaxUb = 20480;
 constexpr uint32_t kMaxProbe = 96;
 constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
@@ -303,14 +303,16 @@ __device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, 
 
 // ---- 4b. block hash / span-bitmap bins --------------------------------------
 // Bucketed ORDER-PRESERVING hash: bucket b = floor((c - lo) * nb / span) is
-// monotone in c, so buckets are mutually ordered; each bucket has 8 slots
-// (mean load 4), claimed by atomicCAS scanning from slot 0 (the scan order
-// makes duplicates meet).  A full bucket spills to a small monotone
-// linear-probing overflow table.  Emission: per-thread runs of buckets, a
-// block scan of their counts, an 8-input Batcher network sorts each bucket
-// in registers, and the (few) overflow elements are merged by rank:
-//   main v at bucket b, index j : prefix(b) + j + #(overflow < v)
-//   overflow x (i-th smallest)  : prefix(b_x) + #(bucket b_x < x) + i
+// monotone in c, so buckets are mutually ordered.  Each bucket has 8 slots
+// (mean load 4) and a fill counter: an insert is one smem atomicAdd on the
+// counter and one store - no probing, no CAS, no lane divergence; duplicates
+// are dropped at emission.  Products arriving at a full bucket go to a small
+// monotone linear-probing overflow table (atomicCAS, duplicate-free).
+// Emission: per-thread runs of buckets; each bucket is sorted in registers by
+// an 8-input Batcher network, merged with its (rare) overflow elements and
+// deduplicated; a block scan of the per-thread unique counts gives the output
+// offsets (the sort is repeated in the write pass instead of keeping 8
+// registers per bucket live across the scan).
 __device__ __forceinline__ void cswap(idx_t& a, idx_t& b) {
     const idx_t x = min(a, b), y = max(a, b);
     a = x;
@@ -324,18 +326,60 @@ __device__ __forceinline__ void sort8(idx_t (&v)[8]) {  // Batcher odd-even merg
     cswap(v[2], v[4]); cswap(v[3], v[5]);
     cswap(v[1], v[2]); cswap(v[3], v[4]); cswap(v[5], v[6]);
 }
-__device__ __forceinline__ uint32_t lower_bound_smem(const idx_t* a, uint32_t n, idx_t key) {
-    uint32_t lo = 0, hi = n;
-    while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (a[mid] < key) lo = mid + 1; else hi = mid;
-    }
-    return lo;
-}
 
 constexpr uint32_t kOvSlack = 128;
 
-// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] | ovt[OVS+kOvSlack] | ovs[OVS]
+// Sorted bucket b (kEmpty-padded) -> emit (or count when out == nullptr) its
+// distinct values merged with the sorted overflow run ovs[oi, oe).
+__device__ __forceinline__ uint32_t bucket_emit(const idx_t* tab, const uint32_t* cnt, uint32_t b,
+                                                const idx_t* ovs, uint32_t oi, uint32_t oe,
+                                                idx_t* __restrict__ out) {
+    const uint32_t n = min(cnt[b], 8u);
+    const uint4* p4 = reinterpret_cast<const uint4*>(tab + b * 8);
+    const uint4 x = p4[0], y = p4[1];
+    idx_t v[8] = {x.x, x.y, x.z, x.w, y.x, y.y, y.z, y.w};
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+        if (uint32_t(j) >= n) v[j] = kEmpty;
+    sort8(v);
+    uint32_t m = 0;
+    idx_t prev = kEmpty;
+    if (oi == oe) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            if (v[j] != kEmpty && v[j] != prev) {
+                if (out) out[m] = v[j];
+                ++m;
+            }
+            prev = v[j];
+        }
+        return m;
+    }
+    // merge with the overflow run (both sorted), dropping duplicates
+    int j = 0;
+    uint32_t q = oi;
+    for (;;) {
+        const idx_t a = j < 8 ? v[j] : kEmpty;
+        const idx_t c = q < oe ? ovs[q] : kEmpty;
+        if (a == kEmpty && c == kEmpty) break;
+        idx_t t;
+        if (a <= c) {
+            t = a;
+            ++j;
+        } else {
+            t = c;
+            ++q;
+        }
+        if (t != prev) {
+            if (out) out[m] = t;
+            ++m;
+            prev = t;
+        }
+    }
+    return m;
+}
+
+// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] | cnt[MAXB] | ovt[OVS+kOvSlack] | ovs[OVS]
 template <int THREADS, uint32_t MAXB, uint32_t OVS, uint32_t BATCH, int MINB, int FLATU>
 __global__ void __launch_bounds__(THREADS, MINB)
 hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
@@ -347,11 +391,11 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
     idx_t* tab = reinterpret_cast<idx_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
-    idx_t* ovt = tab + MAXB * 8;
+    uint32_t* bcnt = tab + MAXB * 8;
+    idx_t* ovt = bcnt + MAXB;
     idx_t* ovs = ovt + OVS + kOvSlack;
     __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_base[THREADS];
     __shared__ uint32_t s_item, s_flag, s_novf;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
     for (;;) {
@@ -389,22 +433,18 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         }
         const uint32_t ovn = min(max(u / 16, 64u), OVS);
         const uint32_t ovslots = ovn + kOvSlack;
-        fill_words(tab, nb * 8, kEmpty, THREADS);
+        fill_words(bcnt, nb, 0u, THREADS);
         fill_words(ovt, ovslots, kEmpty, THREADS);
         __syncthreads();
         const uint64_t bscale = (uint64_t(nb) << 32) / span;
         const uint64_t oscale = (uint64_t(ovn) << 32) / span;
         block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
             const uint64_t d = uint64_t(c - clo);
-            idx_t* bk = tab + uint32_t((d * bscale) >> 32) * 8;
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                const idx_t cur = bk[k];
-                if (cur == c) return;
-                if (cur == kEmpty) {
-                    const idx_t old = atomicCAS(&bk[k], kEmpty, c);
-                    if (old == kEmpty || old == c) return;
-                }
+            const uint32_t b = uint32_t((d * bscale) >> 32);
+            const uint32_t slot = atomicAdd(&bcnt[b], 1u);
+            if (slot < 8) {
+                tab[b * 8 + slot] = c;
+                return;
             }
             // bucket full: overflow table (monotone linear probing, no wrap)
             uint32_t h = uint32_t((d * oscale) >> 32);
@@ -432,49 +472,39 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         }
         const uint32_t novf = s_novf;
         if (novf) emit_table_ranked<NW>(ovt, ovslots, ovs, s_w);  // sorted overflow -> ovs (smem)
-        // main buckets: thread t owns buckets [t*k, (t+1)*k)
+        // thread t owns buckets [t*k, (t+1)*k); ovs runs located by bucket
         const uint32_t k = (nb + THREADS - 1) / THREADS;
         const uint32_t b0 = threadIdx.x * k, b1 = min(b0 + k, nb);
-        uint64_t cnt = 0;
-        for (uint32_t b = b0; b < b1; ++b) {
-            const uint4* p4 = reinterpret_cast<const uint4*>(tab + b * 8);
-            const uint4 x = p4[0], y = p4[1];
-            cnt += (x.x != kEmpty) + (x.y != kEmpty) + (x.z != kEmpty) + (x.w != kEmpty) +
-                   (y.x != kEmpty) + (y.y != kEmpty) + (y.z != kEmpty) + (y.w != kEmpty);
-        }
-        uint64_t total_main;
-        uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(cnt, s_scan, &total_main));
-        s_base[threadIdx.x] = pos;
-        for (uint32_t b = b0; b < b1; ++b) {
-            const uint4* p4 = reinterpret_cast<const uint4*>(tab + b * 8);
-            const uint4 x = p4[0], y = p4[1];
-            idx_t v[8] = {x.x, x.y, x.z, x.w, y.x, y.y, y.z, y.w};
-            sort8(v);
-#pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                if (v[j] != kEmpty) {
-                    const uint32_t extra = novf ? lower_bound_smem(ovs, novf, v[j]) : 0u;
-                    out[pos + extra] = v[j];
-                    ++pos;
-                }
-            }
-        }
+        auto obucket = [&](uint32_t i) { return uint32_t((uint64_t(ovs[i] - clo) * bscale) >> 32); };
+        uint32_t o0 = 0;
         if (novf) {
-            __syncthreads();  // s_base complete
-            for (uint32_t i = threadIdx.x; i < novf; i += THREADS) {
-                const idx_t xv = ovs[i];
-                const uint32_t b = uint32_t((uint64_t(xv - clo) * bscale) >> 32);
-                const uint32_t owner = b / k;
-                uint32_t p = s_base[owner];
-                for (uint32_t bb = owner * k; bb <= b; ++bb)
-                    for (int j = 0; j < 8; ++j) {
-                        const idx_t w = tab[bb * 8 + j];
-                        p += (w != kEmpty) && (bb < b || w < xv);
-                    }
-                out[p + i] = xv;
+            uint32_t lo = 0, hi = novf;
+            while (lo < hi) {
+                const uint32_t mid = (lo + hi) >> 1;
+                if (obucket(mid) < b0) lo = mid + 1; else hi = mid;
             }
+            o0 = lo;
         }
-        if (threadIdx.x == 0) counts[r] = uint32_t(total_main) + novf;
+        uint64_t cnt = 0;
+        uint32_t oi = o0;
+        for (uint32_t b = b0; b < b1; ++b) {
+            uint32_t oe = oi;
+            if (bcnt[b] > 8)
+                while (oe < novf && obucket(oe) == b) ++oe;
+            cnt += bucket_emit(tab, bcnt, b, ovs, oi, oe, nullptr);
+            oi = oe;
+        }
+        uint64_t total;
+        uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(cnt, s_scan, &total));
+        oi = o0;
+        for (uint32_t b = b0; b < b1; ++b) {
+            uint32_t oe = oi;
+            if (bcnt[b] > 8)
+                while (oe < novf && obucket(oe) == b) ++oe;
+            pos += bucket_emit(tab, bcnt, b, ovs, oi, oe, out + pos);
+            oi = oe;
+        }
+        if (threadIdx.x == 0) counts[r] = uint32_t(total);
         __syncthreads();
     }
 }
@@ -730,9 +760,9 @@ __global__ void compact_kernel(const idx_t* __restrict__ scratch, const uint64_t
 constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 constexpr uint32_t kSBatch = 512, kLBatch = 384, kXBatch = 256, kDBatch = 2048;
 constexpr uint32_t kSBuckets = kHashSMaxUb / 4, kLBuckets = kHashLMaxUb / 4, kXBuckets = kHashXMaxUb / 4;
-constexpr uint32_t kSOvs = 128, kLOvs = 384, kXOvs = 1536;
+constexpr uint32_t kSOvs = 128, kLOvs = 384, kXOvs = 1024;
 constexpr size_t hash_smem(uint32_t batch, uint32_t buckets, uint32_t ovs) {
-    return batch * kSegBytes + (buckets * 8 + ovs + kOvSlack + ovs) * sizeof(idx_t);
+    return batch * kSegBytes + (buckets * 9 + ovs + kOvSlack + ovs) * sizeof(idx_t);
 }
 constexpr size_t kSSmem = hash_smem(kSBatch, kSBuckets, kSOvs);
 constexpr size_t kLSmem = hash_smem(kLBatch, kLBuckets, kLOvs);
@@ -742,8 +772,8 @@ constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 
 #define HASH_L hash_bin_kernel<512, kLBuckets, kLOvs, kLBatch, 3, 4>
 #define HASH_X hash_bin_kernel<1024, kXBuckets, kXOvs, kXBatch, 1, 8>
 #define DENSE dense_bin_kernel<1024, kDBatch, 8>
-static_assert(kLSmem + 2 * 1024 + 700 <= 227 * 1024 / 3, "hash-L: 3 blocks per SM");
-static_assert(kXSmem + 4 * 1024 + 700 <= 227 * 1024, "hash-X fits");
+static_assert(3 * (kLSmem + 1024 + 600) <= 228 * 1024, "hash-L: 3 blocks per SM");
+static_assert(kXSmem + 600 <= 227 * 1024, "hash-X fits");
 
 static void ensure_attrs() {
     static int done_dev = -1;
