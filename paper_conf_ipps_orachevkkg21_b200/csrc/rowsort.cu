@@ -38,15 +38,14 @@ namespace spbla {
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int kNumBins = 10;
+constexpr int kNumBins = 12;
 enum {
     BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16,
-    BIN_HASH_S = 6, BIN_HASH_L = 7, BIN_HASH_X = 8, BIN_DENSE = 9
+    BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_DENSE = 11
 };
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 512
-constexpr uint64_t kHashSMaxUb = 2048;
-constexpr uint64_t kHashLMaxUb = 6144;
-constexpr uint64_t kHashXMaxUb = 20480;
+// hash bins: ub limits (each sized so its tables fit the residency below)
+constexpr uint64_t kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480;
 constexpr uint32_t kMaxProbe = 96;
 constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
@@ -58,9 +57,11 @@ __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub <= 128) return BIN_W4;
     if (ub <= 256) return BIN_W8;
     if (ub <= kWarpMaxUb) return BIN_W16;
-    if (ub <= kHashSMaxUb) return BIN_HASH_S;
-    if (ub <= kHashLMaxUb) return BIN_HASH_L;
-    if (ub <= kHashXMaxUb) return BIN_HASH_X;
+    if (ub <= kH1) return BIN_H1;
+    if (ub <= kH2) return BIN_H2;
+    if (ub <= kH3) return BIN_H3;
+    if (ub <= kH4) return BIN_H4;
+    if (ub <= kH5) return BIN_H5;
     return BIN_DENSE;
 }
 
@@ -758,29 +759,39 @@ __global__ void compact_kernel(const idx_t* __restrict__ scratch, const uint64_t
 
 // ------------------------------------------------------------------------------
 constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
-constexpr uint32_t kSBatch = 512, kLBatch = 384, kXBatch = 256, kDBatch = 2048;
-constexpr uint32_t kSBuckets = kHashSMaxUb / 4, kLBuckets = kHashLMaxUb / 4, kXBuckets = kHashXMaxUb / 4;
-constexpr uint32_t kSOvs = 128, kLOvs = 384, kXOvs = 1024;
+// hash bins: <threads, max buckets (= ub limit / 4), overflow slots, descriptor
+// batch, blocks per SM, loads in flight>; smem per block is checked against
+// the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
+constexpr uint32_t kDBatch = 2048;
 constexpr size_t hash_smem(uint32_t batch, uint32_t buckets, uint32_t ovs) {
     return batch * kSegBytes + (buckets * 9 + ovs + kOvSlack + ovs) * sizeof(idx_t);
 }
-constexpr size_t kSSmem = hash_smem(kSBatch, kSBuckets, kSOvs);
-constexpr size_t kLSmem = hash_smem(kLBatch, kLBuckets, kLOvs);
-constexpr size_t kXSmem = hash_smem(kXBatch, kXBuckets, kXOvs);
+#define HBIN(NAME, T, UB, OVS, BATCH, PERSM, U)                                                    \
+    constexpr int NAME##_T = T, NAME##_PERSM = PERSM;                                             \
+    constexpr size_t NAME##_SMEM = hash_smem(BATCH, uint32_t(UB / 4), OVS);                      \
+    static_assert(PERSM * (NAME##_SMEM + 1024 + 600) <= 228 * 1024, #NAME " residency");          \
+    static_assert(PERSM * T <= 2048, #NAME " threads");
+HBIN(H1, 128, kH1, 64, 256, 12, 4)
+HBIN(H2, 256, kH2, 128, 512, 6, 4)
+HBIN(H3, 256, kH3, 256, 384, 5, 4)
+HBIN(H4, 512, kH4, 512, 256, 2, 4)
+HBIN(H5, 1024, kH5, 1024, 256, 1, 8)
+#define HASH1 hash_bin_kernel<128, uint32_t(kH1 / 4), 64, 256, 12, 4>
+#define HASH2 hash_bin_kernel<256, uint32_t(kH2 / 4), 128, 512, 6, 4>
+#define HASH3 hash_bin_kernel<256, uint32_t(kH3 / 4), 256, 384, 5, 4>
+#define HASH4 hash_bin_kernel<512, uint32_t(kH4 / 4), 512, 256, 2, 4>
+#define HASH5 hash_bin_kernel<1024, uint32_t(kH5 / 4), 1024, 256, 1, 8>
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
-#define HASH_S hash_bin_kernel<256, kSBuckets, kSOvs, kSBatch, 6, 4>
-#define HASH_L hash_bin_kernel<512, kLBuckets, kLOvs, kLBatch, 3, 4>
-#define HASH_X hash_bin_kernel<1024, kXBuckets, kXOvs, kXBatch, 1, 8>
 #define DENSE dense_bin_kernel<1024, kDBatch, 8>
-static_assert(3 * (kLSmem + 1024 + 600) <= 228 * 1024, "hash-L: 3 blocks per SM");
-static_assert(kXSmem + 600 <= 227 * 1024, "hash-X fits");
 
 static void ensure_attrs() {
     static int done_dev = -1;
     if (done_dev == ctx().device) return;
-    CUDA_CHECK(cudaFuncSetAttribute(HASH_S, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kSSmem)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH_L, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kLSmem)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH_X, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kXSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH1, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H1_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH2, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H2_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH3, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H3_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH4, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H4_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH5, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H5_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(DENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDSmem)));
     done_dev = ctx().device;
 }
@@ -799,13 +810,13 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    // meta: hist[10] binoff[11] cursor[10] work[6] ovf[2]
+    // meta: hist[12] binoff[13] cursor[12] work[8] ovf[2]
     DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
-    uint32_t* binoff = meta.p + 10;
-    uint32_t* cursor = meta.p + 21;
-    uint32_t* work = meta.p + 31;
-    uint32_t* ovf = meta.p + 38;  // ovf[0] = 0 (list start), ovf[1] = count
+    uint32_t* binoff = meta.p + 12;
+    uint32_t* cursor = meta.p + 25;
+    uint32_t* work = meta.p + 37;
+    uint32_t* ovf = meta.p + 45;  // ovf[0] = 0 (list start), ovf[1] = count
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
     const unsigned gb = (unsigned)std::min<uint64_t>(ceil_div(nrows, 256), uint64_t(nsm) * 8);
     bin_count_kernel<<<gb, 256, 0, st>>>(ub, nrows, ncols, cap.p, bin.p, counts.p, hist);
@@ -834,21 +845,20 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DENSE<<<nsm, 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols, scratch.p, soff.p,
                                      counts.p, work);
     ktime_end(t);
-    t = ktime_begin("hash_x", st);
-    HASH_X<<<nsm, 1024, kXSmem, st>>>(src, rows.p, binoff + BIN_HASH_X, ub, range, ncols, scratch.p, soff.p,
-                                      counts.p, work + 1, ovf_rows.p, ovf);
+#define LAUNCH_HASH(K, NAME, BIN, W)                                                                  \
+    t = ktime_begin(#NAME, st);                                                                         \
+    K<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, rows.p, binoff + BIN, ub, range, ncols, scratch.p, \
+                                                         soff.p, counts.p, work + W, ovf_rows.p, ovf);  \
     ktime_end(t);
-    t = ktime_begin("hash_l", st);
-    HASH_L<<<nsm * 3, 512, kLSmem, st>>>(src, rows.p, binoff + BIN_HASH_L, ub, range, ncols, scratch.p, soff.p,
-                                         counts.p, work + 2, ovf_rows.p, ovf);
-    ktime_end(t);
-    t = ktime_begin("hash_s", st);
-    HASH_S<<<nsm * 6, 256, kSSmem, st>>>(src, rows.p, binoff + BIN_HASH_S, ub, range, ncols, scratch.p, soff.p,
-                                         counts.p, work + 3, ovf_rows.p, ovf);
-    ktime_end(t);
+    LAUNCH_HASH(HASH5, H5, BIN_H5, 1)
+    LAUNCH_HASH(HASH4, H4, BIN_H4, 2)
+    LAUNCH_HASH(HASH3, H3, BIN_H3, 3)
+    LAUNCH_HASH(HASH2, H2, BIN_H2, 4)
+    LAUNCH_HASH(HASH1, H1, BIN_H1, 5)
+#undef LAUNCH_HASH
     // rows whose hash probes ran long: bitmap path
-    DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 4);
-    count_launch(5);
+    DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 6);
+    count_launch(7);
     check_launch("block bins");
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
     t = ktime_begin("warp_bins", st);
@@ -879,11 +889,11 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
 }
 
 void engine_thresholds(uint64_t* out, uint32_t* n) {
-    // ub upper limits of bins W1, W2, W4, W8, W16, HASH_S, HASH_L, HASH_X (DENSE above)
-    const uint64_t t[8] = {32, 64, 128, 256, kWarpMaxUb, kHashSMaxUb, kHashLMaxUb, kHashXMaxUb};
-    const uint32_t k = *n < 8 ? *n : 8;
+    // ub upper limits of bins W1, W2, W4, W8, W16, H1..H5 (DENSE above)
+    const uint64_t t[10] = {32, 64, 128, 256, kWarpMaxUb, kH1, kH2, kH3, kH4, kH5};
+    const uint32_t k = *n < 10 ? *n : 10;
     for (uint32_t i = 0; i < k; ++i) out[i] = t[i];
-    *n = 8;
+    *n = 10;
 }
 
 }  // namespace spbla
