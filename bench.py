@@ -191,11 +191,16 @@ def main():
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % torch.cuda.device_count()
     torch.cuda.set_device(local)
     import torch.distributed as dist
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        # NCCL over NVLink; SPBLA_DIST_BACKEND=gloo runs several ranks on one GPU (testing only)
+        backend = os.environ.get("SPBLA_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        else:
+            dist.init_process_group(backend)
     import paper_conf_ipps_orachevkkg21_b200 as sp
     from paper_conf_ipps_orachevkkg21_b200 import dist as spdist
     sp.Initialize(local)
@@ -223,10 +228,7 @@ def main():
         A = Afull
     ub = ub_full[r0:r1]
     products_local = int(ub.sum())
-    prod_t = torch.tensor([products_local], dtype=torch.int64, device="cuda")
-    if world > 1:
-        dist.all_reduce(prod_t)
-    products = int(prod_t)
+    products = spdist.allreduce_int(products_local) if world > 1 else products_local
     nnzA = A.nvals
     log(f"[rank {rank}] setup {time.time() - t0:.1f}s: n={n} rows[{r0},{r1}) nnzA={nnzA} "
         f"products(total)={products}")
@@ -274,7 +276,8 @@ def main():
               ("mxm_ub", "warp_bins", "H1", "H2", "H3", "H4", "H5", "dense", "compact")}
     sp.set_kernel_timing(False)
     peak_mem = sp.memory_stats()[1]
-    tot = torch.tensor([sum(step_ms), peak_mem, nnzC_local, launches], dtype=torch.float64, device="cuda")
+    red_dev = "cpu" if world > 1 and dist.get_backend() == "gloo" else "cuda"
+    tot = torch.tensor([sum(step_ms), peak_mem, nnzC_local, launches], dtype=torch.float64, device=red_dev)
     if world > 1:
         mx = tot.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
@@ -351,7 +354,7 @@ def main():
             torch.cuda.synchronize()
             if i:
                 e2e_ms.append(1e3 * (time.perf_counter() - t))
-        et = torch.tensor([sum(e2e_ms) / len(e2e_ms)], dtype=torch.float64, device="cuda")
+        et = torch.tensor([sum(e2e_ms) / len(e2e_ms)], dtype=torch.float64, device=red_dev)
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e = {"value": products / (float(et) * 1e-3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,

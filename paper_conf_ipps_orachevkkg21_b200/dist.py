@@ -42,6 +42,10 @@ def allgather_csr(rowptr: torch.Tensor, colidx: torch.Tensor, group=None):
     Blocks are padded to the largest one for the collective."""
     world = dist.get_world_size(group)
     dev = rowptr.device
+    if dev.type == "cuda" and dist.get_backend(group) == "gloo":
+        # gloo path (CPU tests / single-GPU multi-rank runs): collective on host copies
+        blocks = allgather_csr(rowptr.cpu(), colidx.cpu(), group)
+        return [(nr, rp.to(dev), ci.to(dev), nz) for nr, rp, ci, nz in blocks]
     nrows = rowptr.numel() - 1
     nnz = colidx.numel()
     sizes = torch.tensor([nrows, nnz], dtype=torch.int64, device=dev)
@@ -90,6 +94,14 @@ class CudaOps:
         return C
 
 
+def allreduce_int(x: int, group=None, op=dist.ReduceOp.SUM, device=None) -> int:
+    """All-reduce of one integer (host tensor for gloo, device tensor for NCCL)."""
+    dev = "cpu" if dist.get_backend(group) == "gloo" else (device or "cuda")
+    t = torch.tensor([x], dtype=torch.int64, device=dev)
+    dist.all_reduce(t, op=op, group=group)
+    return int(t)
+
+
 def gather_rows(ops, M_local, nrows_total, ncols, group=None):
     rp, ci = ops.csr(M_local)
     blocks = allgather_csr(rp, ci, group)
@@ -108,16 +120,14 @@ def distributed_closure(ops, C_local, n, group=None, max_iters=10_000):
     all-gathers the C shards (B = C), updates the local rows, and all-reduces
     nnz to detect the fixed point.  Returns (C_local, iterations)."""
     dev = ops.csr(C_local)[0].device
-    prev = torch.tensor([ops.nvals(C_local)], dtype=torch.int64, device=dev)
-    dist.all_reduce(prev, group=group)
+    prev = allreduce_int(ops.nvals(C_local), group, device=dev)
     it = 0
     while it < max_iters:
         B = gather_rows(ops, C_local, n, n, group)
         C_local = ops.mxm(C_local, C_local, B, True)
         it += 1
-        cur = torch.tensor([ops.nvals(C_local)], dtype=torch.int64, device=dev)
-        dist.all_reduce(cur, group=group)
-        if int(cur) == int(prev):
+        cur = allreduce_int(ops.nvals(C_local), group, device=dev)
+        if cur == prev:
             break
         prev = cur
     return C_local, it

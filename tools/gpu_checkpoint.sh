@@ -1,0 +1,13 @@
+#!/bin/bash
+# One GPU checkpoint: tests, bench (both arms), 2-rank smoke on one GPU,
+# ncu launch list + one full capture of the top kernel.  Output: gpurun_out/ckpt/
+cd "$(dirname "$0")/.."
+O=gpurun_out/ckpt; mkdir -p $O
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.used --format=csv > $O/gpu.txt
+timeout 1200 python -m pytest tests -m gpu -q > $O/pytest_gpu.txt 2>&1; tail -2 $O/pytest_gpu.txt
+timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; cut -c1-200 $O/bench.json
+timeout 600 python bench.py --impl reference > $O/bench_ref.json 2> $O/bench_ref.err; cut -c1-160 $O/bench_ref.json
+SPBLA_DIST_BACKEND=gloo timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 2 --warmup 3 --workload rmat20_ef16 --no-cpu-baseline > $O/bench_2rank_gloo.json 2> $O/bench_2rank_gloo.err; cut -c1-200 $O/bench_2rank_gloo.json
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_launch_bench.log 2>&1
+timeout 1200 ncu --set full --import-source on --clock-control none -k regex:${TOPK:-hash_bin_kernel} -s ${TOPS:-1} -c 1 -o $O/top python tools/quick_mxm.py 22 32 0.4 0.2 0.2 > $O/ncu_top.log 2>&1
+ls -la $O
