@@ -380,7 +380,8 @@ __device__ __forceinline__ uint32_t bucket_emit(const idx_t* tab, const uint32_t
     return m;
 }
 
-// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] | cnt[MAXB] | ovt[OVS+kOvSlack] | ovs[OVS]
+// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] | cnt[MAXB] | ovt[OVS+kOvSlack] | ovs[OVS+kOvSlack]
+// (ovs holds the sorted overflow elements: at most the table's OVS+kOvSlack slots)
 template <int THREADS, uint32_t MAXB, uint32_t OVS, uint32_t BATCH, int MINB, int FLATU>
 __global__ void __launch_bounds__(THREADS, MINB)
 hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
@@ -764,7 +765,7 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
 constexpr uint32_t kDBatch = 2048;
 constexpr size_t hash_smem(uint32_t batch, uint32_t buckets, uint32_t ovs) {
-    return batch * kSegBytes + (buckets * 9 + ovs + kOvSlack + ovs) * sizeof(idx_t);
+    return batch * kSegBytes + (buckets * 9 + 2 * (ovs + kOvSlack)) * sizeof(idx_t);
 }
 #define HBIN(NAME, T, UB, OVS, BATCH, PERSM, U)                                                    \
     constexpr int NAME##_T = T, NAME##_PERSM = PERSM;                                             \
