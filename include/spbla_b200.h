@@ -88,6 +88,8 @@ spbla_Status spbla_Synchronize(void);
  * since the last spbla_ResetPeakMemory. */
 spbla_Status spbla_GetMemoryStats(uint64_t* current_bytes, uint64_t* peak_bytes);
 spbla_Status spbla_ResetPeakMemory(void);
+/* Bytes the stream-ordered pool has reserved from the device / hands out. */
+spbla_Status spbla_GetPoolStats(uint64_t* reserved_bytes, uint64_t* used_bytes);
 const char* spbla_GetLastErrorMessage(void);
 const char* spbla_GetVersion(void);
 /* Number of kernels the library has launched since the last reset (the

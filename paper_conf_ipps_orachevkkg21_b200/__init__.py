@@ -86,6 +86,13 @@ def memory_stats():
     return int(cur.value), int(peak.value)
 
 
+def pool_stats():
+    """(reserved, used) bytes of the library's stream-ordered pool."""
+    r, u = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(_lib().spbla_GetPoolStats(ctypes.byref(r), ctypes.byref(u)), "spbla_GetPoolStats")
+    return int(r.value), int(u.value)
+
+
 def reset_peak_memory():
     _check(_lib().spbla_ResetPeakMemory(), "spbla_ResetPeakMemory")
 

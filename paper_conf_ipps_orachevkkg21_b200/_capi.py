@@ -24,6 +24,7 @@ SIGNATURES = {
     "spbla_Synchronize": (_int, []),
     "spbla_GetMemoryStats": (_int, [_pu64, _pu64]),
     "spbla_ResetPeakMemory": (_int, []),
+    "spbla_GetPoolStats": (_int, [_pu64, _pu64]),
     "spbla_GetLastErrorMessage": (ctypes.c_char_p, []),
     "spbla_GetVersion": (ctypes.c_char_p, []),
     "spbla_GetLaunchCount": (_u64, []),

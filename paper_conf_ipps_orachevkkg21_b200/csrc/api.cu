@@ -119,6 +119,17 @@ spbla_Status spbla_GetMemoryStats(uint64_t* cur, uint64_t* peak) {
     });
 }
 
+spbla_Status spbla_GetPoolStats(uint64_t* reserved, uint64_t* used) {
+    return guarded([&] {
+        require_init();
+        uint64_t r = 0, u = 0;
+        CUDA_CHECK(cudaMemPoolGetAttribute(ctx().pool, cudaMemPoolAttrReservedMemCurrent, &r));
+        CUDA_CHECK(cudaMemPoolGetAttribute(ctx().pool, cudaMemPoolAttrUsedMemCurrent, &u));
+        if (reserved) *reserved = r;
+        if (used) *used = u;
+    });
+}
+
 spbla_Status spbla_ResetPeakMemory(void) {
     return guarded([&] { ctx().peak_bytes = ctx().cur_bytes; });
 }
