@@ -129,6 +129,10 @@ struct SegSource {
     const off_t64* __restrict__ brp; const idx_t* __restrict__ bci;
     const off_t64* __restrict__ crp; const idx_t* __restrict__ cci;
     const off_t64* __restrict__ lrp; const idx_t* __restrict__ lst;
+    // MxM: per A entry p the B segment as {ptr lo, ptr hi, len, 0} (written by
+    // the upper-bound pass, so staging a row costs one coalesced load per
+    // segment instead of the dependent aci -> brp chain); may be null
+    const uint4* __restrict__ desc;
 };
 // ub: per-row upper bound of entries (device, nrows).  Installs the result
 // in `out` (nrows x ncols).  dedup=false promises rows are duplicate-free.

@@ -19,7 +19,8 @@ constexpr int kGroup = 8;
 
 __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
                               const off_t64* __restrict__ crp, const idx_t* __restrict__ cci,
-                              uint64_t* __restrict__ ub, uint2* __restrict__ range) {
+                              uint64_t* __restrict__ ub, uint2* __restrict__ range,
+                              uint4* __restrict__ desc) {
     const unsigned g = threadIdx.x & (kGroup - 1);
     const size_t ngroups = (size_t(gridDim.x) * blockDim.x) / kGroup;
     // warp-uniform loop: every lane of a warp runs the same trip count
@@ -34,7 +35,10 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
             e = A.rowptr[r + 1];
             for (off_t64 p = b + g; p < e; p += kGroup) {
                 idx_t k = A.colidx[p];
-                s += brp[k + 1] - brp[k];
+                const off_t64 x = brp[k], y = brp[k + 1];
+                s += y - x;
+                const uint64_t ptr = reinterpret_cast<uint64_t>(bci + x);
+                desc[p] = make_uint4(uint32_t(ptr), uint32_t(ptr >> 32), uint32_t(y - x), 0u);
             }
         }
 #pragma unroll
@@ -86,12 +90,13 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     }
     DevBuf<uint64_t> ub(m);
     DevBuf<uint2> range(m);
+    DevBuf<uint4> desc(A->nnz);
     const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
                                                        uint64_t(ctx().num_sms) * 16);
     const off_t64* crp = accumulate ? C->rowptr : nullptr;
     int tk = ktime_begin("mxm_ub", ctx().stream);
     mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, crp,
-                                                  accumulate ? C->colidx : nullptr, ub.p, range.p);
+                                                  accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p);
     ktime_end(tk);
     count_launch();
     check_launch("mxm_ub_kernel");
@@ -104,6 +109,7 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     src.bci = B->colidx;
     src.crp = crp;
     src.cci = accumulate ? C->colidx : nullptr;
+    src.desc = desc.p;
     // the engine writes fresh storage and only then installs it into C, so
     // C may alias A and/or B
     Matrix tmp;

@@ -85,6 +85,11 @@ __device__ __forceinline__ const idx_t* get_seg(const SegSource& s, idx_t r, uin
         }
         --j;
     }
+    if (s.desc) {
+        const uint4 d = s.desc[s.arp[r] + j];
+        len = d.z;
+        return reinterpret_cast<const idx_t*>((uint64_t(d.y) << 32) | d.x);
+    }
     idx_t k = s.aci[s.arp[r] + j];
     off_t64 b = s.brp[k];
     len = uint32_t(s.brp[k + 1] - b);
