@@ -74,11 +74,12 @@ def load():
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(LIB):
+    lib_path = os.environ.get("SPBLA_LIB_PATH", LIB)  # debug builds (tools/probe.sh) only
+    if not os.path.exists(lib_path):
         raise ImportError(
             f"{LIB} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
             "(the CUDA library is the only implementation; there is no fallback)")
-    lib = ctypes.CDLL(LIB)
+    lib = ctypes.CDLL(lib_path)
     for name, (res, args) in SIGNATURES.items():
         fn = getattr(lib, name)
         fn.restype = res

@@ -38,6 +38,32 @@ namespace spbla {
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
+
+#ifdef SPBLA_PROBE
+// Debug-only phase timing (built into a separate .so by tools/probe.sh):
+// block 0, thread 0 prints per-phase nanoseconds for its first rows.
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__shared__ unsigned long long s_probe_ext[12];
+#define PROBE_DECL uint32_t probe_rows = 0;
+#define PROBE(i) do { if (threadIdx.x == 0) s_probe_ext[i] = gtimer(); } while (0)
+#define PROBE_PRINT(tag, u, ns)                                                                      \
+    do {                                                                                           \
+        if (blockIdx.x == 0 && threadIdx.x == 0 && probe_rows++ < 24)                              \
+            printf("%s u=%u nseg=%u meta=%llu fill=%llu stage=%llu prod=%llu ovf=%llu cnt=%llu emit=%llu\n", tag, \
+                   u, ns, s_probe_ext[1] - s_probe_ext[0], s_probe_ext[2] - s_probe_ext[1],                \
+                   s_probe_ext[3] - s_probe_ext[2], s_probe_ext[4] - s_probe_ext[3],                   \
+                   s_probe_ext[5] - s_probe_ext[4], s_probe_ext[6] - s_probe_ext[5],                   \
+                   s_probe_ext[7] - s_probe_ext[6]);                                                  \
+    } while (0)
+#else
+#define PROBE_DECL
+#define PROBE(i) do {} while (0)
+#define PROBE_PRINT(tag, u, ns) do {} while (0)
+#endif
 constexpr int kNumBins = 12;
 enum {
     BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16,
@@ -179,6 +205,9 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, cons
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
         uint32_t ns;
         const uint32_t total = stage_segments<THREADS>(s, r, s0, min(batch, nseg - s0), sd_ptr, sd_end, s_scan, &ns);
+#ifdef SPBLA_PROBE
+        if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
+#endif
         for (uint32_t base = wib * CH; base < total; base += NW * CH) {
             uint32_t lo = 0, hi = ns - 1;  // segment holding product `base`
             while (lo < hi) {
@@ -337,16 +366,18 @@ constexpr uint32_t kOvSlack = 128;
 
 // Sorted bucket b (kEmpty-padded) -> emit (or count when out == nullptr) its
 // distinct values merged with the sorted overflow run ovs[oi, oe).
-__device__ __forceinline__ uint32_t bucket_emit(const idx_t* tab, const uint32_t* cnt, uint32_t b,
-                                                const idx_t* ovs, uint32_t oi, uint32_t oe,
+__device__ __forceinline__ uint32_t bucket_emit(const uint16_t* tab, const uint32_t* cnt, uint32_t b,
+                                                idx_t base, const idx_t* ovs, uint32_t oi, uint32_t oe,
                                                 idx_t* __restrict__ out) {
     const uint32_t n = min(cnt[b], 8u);
-    const uint4* p4 = reinterpret_cast<const uint4*>(tab + b * 8);
-    const uint4 x = p4[0], y = p4[1];
-    idx_t v[8] = {x.x, x.y, x.z, x.w, y.x, y.y, y.z, y.w};
+    const uint4 w = reinterpret_cast<const uint4*>(tab)[b];  // 8 x 16-bit offsets
+    const uint32_t q4[4] = {w.x, w.y, w.z, w.w};
+    idx_t v[8];
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-        if (uint32_t(j) >= n) v[j] = kEmpty;
+    for (int i = 0; i < 4; ++i) {
+        v[2 * i] = uint32_t(2 * i) < n ? base + (q4[i] & 0xFFFFu) : kEmpty;
+        v[2 * i + 1] = uint32_t(2 * i + 1) < n ? base + (q4[i] >> 16) : kEmpty;
+    }
     sort8(v);
     uint32_t m = 0;
     idx_t prev = kEmpty;
@@ -385,7 +416,10 @@ __device__ __forceinline__ uint32_t bucket_emit(const idx_t* tab, const uint32_t
     return m;
 }
 
-// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] | cnt[MAXB] | ovt[OVS+kOvSlack] | ovs[OVS+kOvSlack]
+// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] u16 | cnt[MAXB] | ovt[OVS+kOvSlack] | ovs[OVS+kOvSlack]
+// Bucket b = floor((c - lo) / W) (W = ceil(span / nb) <= 65535, computed with
+// an exact 48-bit reciprocal), each slot the 16-bit offset c - lo - b*W:
+// 20 bytes per bucket of mean load 4, so ~5 bytes of smem per product.
 // (ovs holds the sorted overflow elements: at most the table's OVS+kOvSlack slots)
 template <int THREADS, uint32_t MAXB, uint32_t OVS, uint32_t BATCH, int MINB, int FLATU>
 __global__ void __launch_bounds__(THREADS, MINB)
@@ -397,14 +431,16 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
-    idx_t* tab = reinterpret_cast<idx_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
-    uint32_t* bcnt = tab + MAXB * 8;
+    uint16_t* tab = reinterpret_cast<uint16_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
+    uint32_t* bmw = reinterpret_cast<uint32_t*>(tab);  // bitmap-mode view: MAXB * 5 words
+    uint32_t* bcnt = reinterpret_cast<uint32_t*>(tab + MAXB * 8);
     idx_t* ovt = bcnt + MAXB;
     idx_t* ovs = ovt + OVS + kOvSlack;
     __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
     __shared__ uint32_t s_item, s_flag, s_novf;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
+    PROBE_DECL
     for (;;) {
         if (threadIdx.x == 0) {
             s_item = lo_i + atomicAdd(work, 1u);
@@ -414,6 +450,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         __syncthreads();
         const uint32_t item = s_item;
         if (item >= hi_i) break;
+        PROBE(0);
         const idx_t r = rows[item];
         const uint32_t u = uint32_t(ub[r]);
         uint32_t clo = 0, chi = ncols - 1;
@@ -423,34 +460,45 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             chi = rg.y;
         }
         const uint64_t span = uint64_t(chi) - clo + 1;
-        const uint32_t nb = min(max((u + 3) / 4, 1u), MAXB);
+        // nb buckets of width W <= 65535 (16-bit offsets); too wide a span for the
+        // table goes to the bitmap bin
+        const uint64_t nbw = (span + 65534) / 65535;
+        const uint32_t nb = uint32_t(min(max(max(uint64_t((u + 3) / 4), nbw), uint64_t(1)), uint64_t(MAXB)));
         const uint64_t words = (span + 31) >> 5;
         idx_t* out = scratch + soff[r];
-        if (words <= 8ull * nb) {  // the span bitmap is no larger than the table
+        if (words <= 5ull * nb) {  // the span bitmap is no larger than the table
             const uint32_t nw = uint32_t(words);
-            fill_words(tab, nw, 0u, THREADS);
+            fill_words(bmw, nw, 0u, THREADS);
             __syncthreads();
             block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
                 const uint32_t d = c - clo;
-                atomicOr(&tab[d >> 5], 1u << (d & 31));
+                atomicOr(&bmw[d >> 5], 1u << (d & 31));
             });
-            const uint32_t n = emit_bitmap<NW>(tab, nw, clo, out, s_w);
+            const uint32_t n = emit_bitmap<NW>(bmw, nw, clo, out, s_w);
             if (threadIdx.x == 0) counts[r] = n;
             continue;  // emit_bitmap ends with a barrier
         }
+        PROBE(1);
+        if (nbw > MAXB) {  // span too wide for 16-bit offsets in this table
+            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            __syncthreads();
+            continue;
+        }
+        const uint32_t W = uint32_t((span + nb - 1) / nb);
+        const uint64_t M16 = ((((uint64_t(1) << 48) + W - 1) / W) << 16);  // ceil(2^48 / W) << 16
         const uint32_t ovn = min(max(u / 16, 64u), OVS);
         const uint32_t ovslots = ovn + kOvSlack;
         fill_words(bcnt, nb, 0u, THREADS);
         fill_words(ovt, ovslots, kEmpty, THREADS);
         __syncthreads();
-        const uint64_t bscale = (uint64_t(nb) << 32) / span;
+        PROBE(2);
         const uint64_t oscale = (uint64_t(ovn) << 32) / span;
         block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
             const uint64_t d = uint64_t(c - clo);
-            const uint32_t b = uint32_t((d * bscale) >> 32);
+            const uint32_t b = uint32_t(__umul64hi(d, M16));  // floor(d / W), exact for W < 2^16
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
             if (slot < 8) {
-                tab[b * 8 + slot] = c;
+                tab[b * 8 + slot] = uint16_t(uint32_t(d) - b * W);
                 return;
             }
             // bucket full: overflow table (monotone linear probing, no wrap)
@@ -477,12 +525,13 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             __syncthreads();  // everyone has read s_flag / s_item before reuse
             continue;
         }
+        PROBE(4);
         const uint32_t novf = s_novf;
         if (novf) emit_table_ranked<NW>(ovt, ovslots, ovs, s_w);  // sorted overflow -> ovs (smem)
         // thread t owns buckets [t*k, (t+1)*k); ovs runs located by bucket
         const uint32_t k = (nb + THREADS - 1) / THREADS;
         const uint32_t b0 = threadIdx.x * k, b1 = min(b0 + k, nb);
-        auto obucket = [&](uint32_t i) { return uint32_t((uint64_t(ovs[i] - clo) * bscale) >> 32); };
+        auto obucket = [&](uint32_t i) { return uint32_t(__umul64hi(uint64_t(ovs[i] - clo), M16)); };
         uint32_t o0 = 0;
         if (novf) {
             uint32_t lo = 0, hi = novf;
@@ -498,21 +547,25 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             uint32_t oe = oi;
             if (bcnt[b] > 8)
                 while (oe < novf && obucket(oe) == b) ++oe;
-            cnt += bucket_emit(tab, bcnt, b, ovs, oi, oe, nullptr);
+            cnt += bucket_emit(tab, bcnt, b, clo + b * W, ovs, oi, oe, nullptr);
             oi = oe;
         }
+        PROBE(5);
         uint64_t total;
         uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(cnt, s_scan, &total));
+        PROBE(6);
         oi = o0;
         for (uint32_t b = b0; b < b1; ++b) {
             uint32_t oe = oi;
             if (bcnt[b] > 8)
                 while (oe < novf && obucket(oe) == b) ++oe;
-            pos += bucket_emit(tab, bcnt, b, ovs, oi, oe, out + pos);
+            pos += bucket_emit(tab, bcnt, b, clo + b * W, ovs, oi, oe, out + pos);
             oi = oe;
         }
         if (threadIdx.x == 0) counts[r] = uint32_t(total);
         __syncthreads();
+        PROBE(7);
+        PROBE_PRINT("hash", u, num_segs(src, r));
     }
 }
 
@@ -770,23 +823,25 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
 constexpr uint32_t kDBatch = 2048;
 constexpr size_t hash_smem(uint32_t batch, uint32_t buckets, uint32_t ovs) {
-    return batch * kSegBytes + (buckets * 9 + 2 * (ovs + kOvSlack)) * sizeof(idx_t);
+    return batch * kSegBytes + buckets * (8 * sizeof(uint16_t) + sizeof(uint32_t)) + 2 * (ovs + kOvSlack) * sizeof(idx_t);
 }
 #define HBIN(NAME, T, UB, OVS, BATCH, PERSM, U)                                                    \
-    constexpr int NAME##_T = T, NAME##_PERSM = PERSM;                                             \
+    constexpr int NAME##_T = T, NAME##_PERSM = PERSM, NAME##_U = U;                                \
+    constexpr uint32_t NAME##_B = uint32_t(UB / 4), NAME##_OVS = OVS, NAME##_BATCH = BATCH;        \
     constexpr size_t NAME##_SMEM = hash_smem(BATCH, uint32_t(UB / 4), OVS);                      \
     static_assert(PERSM * (NAME##_SMEM + 1024 + 600) <= 228 * 1024, #NAME " residency");          \
     static_assert(PERSM * T <= 2048, #NAME " threads");
 HBIN(H1, 128, kH1, 64, 256, 12, 4)
-HBIN(H2, 256, kH2, 128, 512, 6, 4)
-HBIN(H3, 256, kH3, 256, 384, 5, 4)
-HBIN(H4, 512, kH4, 512, 256, 2, 4)
-HBIN(H5, 1024, kH5, 1024, 256, 1, 8)
-#define HASH1 hash_bin_kernel<128, uint32_t(kH1 / 4), 64, 256, 12, 4>
-#define HASH2 hash_bin_kernel<256, uint32_t(kH2 / 4), 128, 512, 6, 4>
-#define HASH3 hash_bin_kernel<256, uint32_t(kH3 / 4), 256, 384, 5, 4>
-#define HASH4 hash_bin_kernel<512, uint32_t(kH4 / 4), 512, 256, 2, 4>
-#define HASH5 hash_bin_kernel<1024, uint32_t(kH5 / 4), 1024, 256, 1, 8>
+HBIN(H2, 128, kH2, 128, 256, 12, 4)
+HBIN(H3, 256, kH3, 256, 384, 6, 4)
+HBIN(H4, 256, kH4, 512, 256, 4, 4)
+HBIN(H5, 512, kH5, 512, 256, 2, 8)
+#define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVS, N##_BATCH, N##_PERSM, N##_U>
+#define HASH1 HASHK(H1)
+#define HASH2 HASHK(H2)
+#define HASH3 HASHK(H3)
+#define HASH4 HASHK(H4)
+#define HASH5 HASHK(H5)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
 #define DENSE dense_bin_kernel<1024, kDBatch, 8>
 
