@@ -99,12 +99,12 @@ void spbla_ResetLaunchCount(void);
 /* Per-kernel CUDA-event timing on each kernel's launching stream (bench.py's
  * roofline evidence).  enable != 0 clears previous records and starts
  * recording; spbla_GetKernelTiming sums the recorded launches of the named
- * kernel group ("mxm_ub", "warp_bins", "H1".."H5", "dense", "compact") and
+ * kernel group ("mxm_ub", "warp_bins", "H1".."H6", "dense", "compact") and
  * synchronises on their end events. */
 spbla_Status spbla_SetKernelTiming(int enable);
 spbla_Status spbla_GetKernelTiming(const char* name, double* total_ms, uint64_t* launches);
 /* Upper-bound ("ub") limits of the row engine's bins, ascending: warp bins
- * E=1,2,4,8,16, hash bins H1..H5; rows above the last go to the bitmap bin.  *n: capacity in, count out. */
+ * E=1,2,4,8,16, hash bins H1..H6; rows above the last go to the bitmap bin.  *n: capacity in, count out. */
 spbla_Status spbla_GetEngineThresholds(uint64_t* thresholds, uint32_t* n);
 
 /* ---- matrix life cycle --------------------------- */

@@ -64,14 +64,14 @@ __shared__ unsigned long long s_probe_ext[12];
 #define PROBE(i) do {} while (0)
 #define PROBE_PRINT(tag, u, ns) do {} while (0)
 #endif
-constexpr int kNumBins = 12;
+constexpr int kNumBins = 13;
 enum {
     BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16,
-    BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_DENSE = 11
+    BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_H6, BIN_DENSE = 12
 };
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 512
 // hash bins: ub limits (each sized so its tables fit the residency below)
-constexpr uint64_t kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480;
+constexpr uint64_t kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480, kH6 = 40960;
 constexpr uint32_t kMaxProbe = 96;
 constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
@@ -88,6 +88,7 @@ __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub <= kH3) return BIN_H3;
     if (ub <= kH4) return BIN_H4;
     if (ub <= kH5) return BIN_H5;
+    if (ub <= kH6) return BIN_H6;
     return BIN_DENSE;
 }
 
@@ -836,12 +837,14 @@ HBIN(H2, 128, kH2, 128, 256, 12, 4)
 HBIN(H3, 256, kH3, 256, 384, 6, 4)
 HBIN(H4, 256, kH4, 512, 256, 4, 4)
 HBIN(H5, 512, kH5, 512, 256, 2, 8)
+HBIN(H6, 1024, kH6, 1024, 256, 1, 8)
 #define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVS, N##_BATCH, N##_PERSM, N##_U>
 #define HASH1 HASHK(H1)
 #define HASH2 HASHK(H2)
 #define HASH3 HASHK(H3)
 #define HASH4 HASHK(H4)
 #define HASH5 HASHK(H5)
+#define HASH6 HASHK(H6)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
 #define DENSE dense_bin_kernel<1024, kDBatch, 8>
 
@@ -853,6 +856,7 @@ static void ensure_attrs() {
     CUDA_CHECK(cudaFuncSetAttribute(HASH3, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H3_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(HASH4, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H4_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(HASH5, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H5_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH6, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H6_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(DENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDSmem)));
     done_dev = ctx().device;
 }
@@ -871,13 +875,13 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    // meta: hist[12] binoff[13] cursor[12] work[8] ovf[2]
+    // meta: hist[13] binoff[14] cursor[13] work[9] ovf[2]
     DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
-    uint32_t* binoff = meta.p + 12;
-    uint32_t* cursor = meta.p + 25;
-    uint32_t* work = meta.p + 37;
-    uint32_t* ovf = meta.p + 45;  // ovf[0] = 0 (list start), ovf[1] = count
+    uint32_t* binoff = meta.p + 13;
+    uint32_t* cursor = meta.p + 27;
+    uint32_t* work = meta.p + 40;
+    uint32_t* ovf = meta.p + 49;  // ovf[0] = 0 (list start), ovf[1] = count
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
     const unsigned gb = (unsigned)std::min<uint64_t>(ceil_div(nrows, 256), uint64_t(nsm) * 8);
     bin_count_kernel<<<gb, 256, 0, st>>>(ub, nrows, ncols, cap.p, bin.p, counts.p, hist);
@@ -911,6 +915,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     K<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, rows.p, binoff + BIN, ub, range, ncols, scratch.p, \
                                                          soff.p, counts.p, work + W, ovf_rows.p, ovf);  \
     ktime_end(t);
+    LAUNCH_HASH(HASH6, H6, BIN_H6, 7)
     LAUNCH_HASH(HASH5, H5, BIN_H5, 1)
     LAUNCH_HASH(HASH4, H4, BIN_H4, 2)
     LAUNCH_HASH(HASH3, H3, BIN_H3, 3)
@@ -919,7 +924,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
 #undef LAUNCH_HASH
     // rows whose hash probes ran long: bitmap path
     DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 6);
-    count_launch(7);
+    count_launch(8);
     check_launch("block bins");
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
     t = ktime_begin("warp_bins", st);
@@ -950,11 +955,11 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
 }
 
 void engine_thresholds(uint64_t* out, uint32_t* n) {
-    // ub upper limits of bins W1, W2, W4, W8, W16, H1..H5 (DENSE above)
-    const uint64_t t[10] = {32, 64, 128, 256, kWarpMaxUb, kH1, kH2, kH3, kH4, kH5};
-    const uint32_t k = *n < 10 ? *n : 10;
+    // ub upper limits of bins W1, W2, W4, W8, W16, H1..H6 (DENSE above)
+    const uint64_t t[11] = {32, 64, 128, 256, kWarpMaxUb, kH1, kH2, kH3, kH4, kH5, kH6};
+    const uint32_t k = *n < 11 ? *n : 11;
     for (uint32_t i = 0; i < k; ++i) out[i] = t[i];
-    *n = 10;
+    *n = 11;
 }
 
 }  // namespace spbla

@@ -44,7 +44,7 @@ def sample_rows(ub, n, k=300, seed=0):
     rng = np.random.default_rng(seed)
     ub_h = ub.cpu().numpy()
     heavy = np.argsort(ub_h)[-20:]
-    edges = [0, 1, 33, 65, 129, 257, 513, 1025, 2049, 4097, 8193, 20481, 1 << 62]
+    edges = [0, 1, 33, 65, 129, 257, 513, 1025, 2049, 4097, 8193, 20481, 40961, 1 << 62]
     per_bin = []
     for lo, hi in zip(edges[:-1], edges[1:]):
         idx = np.nonzero((ub_h >= lo) & (ub_h < hi))[0]
