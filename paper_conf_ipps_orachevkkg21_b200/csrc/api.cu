@@ -72,6 +72,15 @@ spbla_Status spbla_Initialize(int device) {
         CUDA_CHECK(cudaDeviceGetDefaultMemPool(&c.pool, device));
         uint64_t thr = UINT64_MAX;  // keep freed blocks cached in the pool
         CUDA_CHECK(cudaMemPoolSetAttribute(c.pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        if (!c.mat_pool) {
+            cudaMemPoolProps props = {};
+            props.allocType = cudaMemAllocationTypePinned;
+            props.handleTypes = cudaMemHandleTypeNone;
+            props.location.type = cudaMemLocationTypeDevice;
+            props.location.id = device;
+            CUDA_CHECK(cudaMemPoolCreate(&c.mat_pool, &props));
+            CUDA_CHECK(cudaMemPoolSetAttribute(c.mat_pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        }
         CUDA_CHECK(cudaMallocHost(&c.host_words, 64));
         c.stream = 0;
         c.device = device;
@@ -84,6 +93,8 @@ spbla_Status spbla_Finalize(void) {
         if (c.device < 0) return;
         CUDA_CHECK(cudaStreamSynchronize(c.stream));
         cudaMemPoolTrimTo(c.pool, 0);
+        if (c.mat_pool) cudaMemPoolDestroy(c.mat_pool);
+        c.mat_pool = nullptr;
         if (c.host_words) cudaFreeHost(c.host_words);
         c.host_words = nullptr;
         c.device = -1;
@@ -123,8 +134,13 @@ spbla_Status spbla_GetPoolStats(uint64_t* reserved, uint64_t* used) {
     return guarded([&] {
         require_init();
         uint64_t r = 0, u = 0;
-        CUDA_CHECK(cudaMemPoolGetAttribute(ctx().pool, cudaMemPoolAttrReservedMemCurrent, &r));
-        CUDA_CHECK(cudaMemPoolGetAttribute(ctx().pool, cudaMemPoolAttrUsedMemCurrent, &u));
+        for (cudaMemPool_t pl : {ctx().pool, ctx().mat_pool}) {
+            uint64_t a = 0, b = 0;
+            CUDA_CHECK(cudaMemPoolGetAttribute(pl, cudaMemPoolAttrReservedMemCurrent, &a));
+            CUDA_CHECK(cudaMemPoolGetAttribute(pl, cudaMemPoolAttrUsedMemCurrent, &b));
+            r += a;
+            u += b;
+        }
         if (reserved) *reserved = r;
         if (used) *used = u;
     });

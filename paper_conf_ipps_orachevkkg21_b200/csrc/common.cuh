@@ -32,7 +32,8 @@ void cuda_check(cudaError_t e, const char* what, const char* file, int line);
 struct Context {
     int device = -1;
     cudaStream_t stream = 0;
-    cudaMemPool_t pool = nullptr;
+    cudaMemPool_t pool = nullptr;      // temporaries (device default pool)
+    cudaMemPool_t mat_pool = nullptr;  // matrix storage (rowptr / colidx of results)
     uint64_t cur_bytes = 0, peak_bytes = 0;
     uint64_t launches = 0;
     int num_sms = kNumSMs;
@@ -43,9 +44,14 @@ struct Context {
 Context& ctx();
 void require_init();
 
-void* dev_alloc(size_t bytes);
+// Two stream-ordered pools: matrix storage (`mat`) and temporaries.  Keeping
+// the long-lived result arrays apart from the scratch of an operation lets a
+// repeated MxM reuse the freed result block exactly instead of fragmenting it
+// with temporaries (a pool miss maps fresh memory: ~60 ms per GB on B200).
+void* dev_alloc(size_t bytes, bool mat = false);
 void dev_free(void* p, size_t bytes);
 // read `n` uint64 words from device memory (synchronises the stream)
+void trace_mark(const char* what);
 void read_words(const uint64_t* dev, uint64_t* host, int n);
 void memset_async(void* p, int v, size_t bytes);
 void copy_async(void* dst, const void* src, size_t bytes, cudaMemcpyKind kind);
@@ -62,11 +68,11 @@ struct DevBuf {
     T* p = nullptr;
     size_t n = 0;
     DevBuf() {}
-    explicit DevBuf(size_t count) { alloc(count); }
-    void alloc(size_t count) {
+    explicit DevBuf(size_t count, bool mat = false) { alloc(count, mat); }
+    void alloc(size_t count, bool mat = false) {
         release();
         n = count;
-        if (count) p = (T*)dev_alloc(count * sizeof(T));
+        if (count) p = (T*)dev_alloc(count * sizeof(T), mat);
     }
     void release() {
         if (p) dev_free(p, n * sizeof(T));
@@ -78,6 +84,8 @@ struct DevBuf {
     DevBuf(const DevBuf&) = delete;
     DevBuf& operator=(const DevBuf&) = delete;
 };
+
+constexpr bool kMat = true;  // DevBuf(count, kMat): storage that becomes a matrix's
 
 // ---- matrix --------------------------------------------------------------
 }  // namespace spbla

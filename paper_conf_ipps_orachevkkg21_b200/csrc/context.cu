@@ -7,6 +7,8 @@
 #include <cstring>
 #include <string>
 #include <vector>
+#include <chrono>
+#include <cstdlib>
 
 namespace spbla {
 
@@ -37,17 +39,19 @@ void check_launch(const char* name) {
     }
 }
 
-void* dev_alloc(size_t bytes) {
+void* dev_alloc(size_t bytes, bool mat) {
     require_init();
     void* p = nullptr;
     if (bytes == 0) return nullptr;
-    cudaError_t e = cudaMallocFromPoolAsync(&p, bytes, g_ctx.pool, g_ctx.stream);
+    cudaMemPool_t pool = mat ? g_ctx.mat_pool : g_ctx.pool;
+    cudaError_t e = cudaMallocFromPoolAsync(&p, bytes, pool, g_ctx.stream);
     if (e != cudaSuccess) {
         (void)cudaGetLastError();
-        // give cached blocks back to the OS and retry once
+        // give cached blocks of both pools back to the OS and retry once
         cudaStreamSynchronize(g_ctx.stream);
         cudaMemPoolTrimTo(g_ctx.pool, 0);
-        e = cudaMallocFromPoolAsync(&p, bytes, g_ctx.pool, g_ctx.stream);
+        cudaMemPoolTrimTo(g_ctx.mat_pool, 0);
+        e = cudaMallocFromPoolAsync(&p, bytes, pool, g_ctx.stream);
         if (e != cudaSuccess) {
             (void)cudaGetLastError();
             char buf[128];
@@ -64,6 +68,27 @@ void dev_free(void* p, size_t bytes) {
     if (!p) return;
     cudaFreeAsync(p, g_ctx.stream);
     g_ctx.cur_bytes -= bytes;
+}
+
+// SPBLA_TRACE=1: synchronise and print wall-clock per phase plus pool
+// reservation (diagnostics only; off by default).
+void trace_mark(const char* what) {
+    static int on = -1;
+    if (on < 0) on = std::getenv("SPBLA_TRACE") != nullptr;
+    if (!on) return;
+    static auto last = std::chrono::steady_clock::now();
+    cudaStreamSynchronize(g_ctx.stream);
+    auto now = std::chrono::steady_clock::now();
+    uint64_t r = 0, u = 0, r2 = 0, u2 = 0;
+    cudaMemPoolGetAttribute(g_ctx.pool, cudaMemPoolAttrReservedMemCurrent, &r);
+    cudaMemPoolGetAttribute(g_ctx.pool, cudaMemPoolAttrUsedMemCurrent, &u);
+    cudaMemPoolGetAttribute(g_ctx.mat_pool, cudaMemPoolAttrReservedMemCurrent, &r2);
+    cudaMemPoolGetAttribute(g_ctx.mat_pool, cudaMemPoolAttrUsedMemCurrent, &u2);
+    r += r2;
+    u += u2;
+    std::fprintf(stderr, "[trace] %-14s %9.3f ms  pool reserved %.2f GB used %.2f GB\n", what,
+                 std::chrono::duration<double, std::milli>(now - last).count(), r / 1e9, u / 1e9);
+    last = now;
 }
 
 void read_words(const uint64_t* dev, uint64_t* host, int n) {
@@ -105,7 +130,7 @@ void matrix_replace(Matrix* m, off_t64* rowptr, size_t rowptr_cap, idx_t* colidx
 }
 
 void matrix_set_empty(Matrix* m) {
-    DevBuf<off_t64> rp(size_t(m->nrows) + 1);
+    DevBuf<off_t64> rp(size_t(m->nrows) + 1, kMat);
     memset_async(rp.p, 0, rp.n * sizeof(off_t64));
     size_t cap = rp.n;
     matrix_replace(m, rp.detach(), cap, nullptr, 0, 0);

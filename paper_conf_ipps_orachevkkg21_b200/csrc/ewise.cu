@@ -197,8 +197,8 @@ void ewise_add(Matrix* C, const Matrix* A, const Matrix* B) {
     uint64_t h;
     read_words(tbase.p + ntiles, &h, 1);
     const uint64_t nnz = m.L - h;
-    DevBuf<off_t64> rp(size_t(A->nrows) + 1);
-    DevBuf<idx_t> ci(nnz);
+    DevBuf<off_t64> rp(size_t(A->nrows) + 1, kMat);
+    DevBuf<idx_t> ci(nnz, kMat);
     merge_write_kernel<<<(unsigned)ntiles, kThreads, 0, ctx().stream>>>(m, tbase.p, ci.p, rp.p);
     count_launch();
     check_launch("merge_write_kernel");

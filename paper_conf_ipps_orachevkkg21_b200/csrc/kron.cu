@@ -56,8 +56,8 @@ void kronecker(Matrix* K, const Matrix* A, const Matrix* B) {
     if (K->nrows != m || K->ncols != n) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "Kronecker: K has the wrong shape");
     if (!K->owned) SPBLA_THROW(SPBLA_STATUS_INVALID_ARGUMENT, "Kronecker: output is a non-owning view");
     const uint64_t nnz = A->nnz * B->nnz;
-    DevBuf<off_t64> rp(m + 1);
-    DevBuf<idx_t> ci(nnz);
+    DevBuf<off_t64> rp(m + 1, kMat);
+    DevBuf<idx_t> ci(nnz, kMat);
     const int nsm = ctx().num_sms;
     unsigned g1 = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(m + 1, 256), uint64_t(nsm) * 16));
     kron_rowptr_kernel<<<g1, 256, 0, ctx().stream>>>(view(A), view(B), B->nnz, rp.p);

@@ -127,9 +127,9 @@ void matrix_build(Matrix* m, const idx_t* rows, const idx_t* cols, uint64_t n, u
     if (h[1]) SPBLA_THROW(SPBLA_STATUS_INDEX_OUT_OF_BOUNDS, "Build: pair outside the matrix");
     const bool presorted = (hints & SPBLA_HINT_SORTED) && (hints & SPBLA_HINT_NO_DUPLICATES);
     if (presorted || n == 0) {
-        DevBuf<off_t64> rp(size_t(nr) + 1);
+        DevBuf<off_t64> rp(size_t(nr) + 1, kMat);
         copy_async(rp.p, bkt.p, rp.n * 8, cudaMemcpyDeviceToDevice);
-        DevBuf<idx_t> ci(n);
+        DevBuf<idx_t> ci(n, kMat);
         copy_async(ci.p, cols, n * sizeof(idx_t), cudaMemcpyDeviceToDevice);
         if (hints & SPBLA_HINT_VALIDATE) validate_csr(rp.p, ci.p, nr, m->ncols, n);
         size_t rc = rp.n, cc = ci.n;
@@ -190,8 +190,8 @@ void matrix_import(Matrix* m, const off_t64* rowptr, const idx_t* colidx, uint64
     if (!m->owned) SPBLA_THROW(SPBLA_STATUS_INVALID_ARGUMENT, "Import: matrix is a non-owning view");
     const bool host = hints & SPBLA_HINT_HOST_MEMORY;
     cudaMemcpyKind k = host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
-    DevBuf<off_t64> rp(size_t(m->nrows) + 1);
-    DevBuf<idx_t> ci(nnz);
+    DevBuf<off_t64> rp(size_t(m->nrows) + 1, kMat);
+    DevBuf<idx_t> ci(nnz, kMat);
     copy_async(rp.p, rowptr, rp.n * 8, k);
     if (nnz) copy_async(ci.p, colidx, nnz * sizeof(idx_t), k);
     if (hints & SPBLA_HINT_VALIDATE) validate_csr(rp.p, ci.p, m->nrows, m->ncols, nnz);
@@ -214,8 +214,8 @@ void matrix_assemble(Matrix* m, uint32_t nblocks, const idx_t* nrows, const off_
         tot_nnz += nnz[b];
     }
     if (tot_rows != m->nrows) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "Assemble: row blocks do not sum to nrows");
-    DevBuf<off_t64> rp(size_t(m->nrows) + 1);
-    DevBuf<idx_t> ci(tot_nnz);
+    DevBuf<off_t64> rp(size_t(m->nrows) + 1, kMat);
+    DevBuf<idx_t> ci(tot_nnz, kMat);
     uint64_t rbase = 0, nbase = 0;
     for (uint32_t b = 0; b < nblocks; ++b) {
         if (nrows[b]) {

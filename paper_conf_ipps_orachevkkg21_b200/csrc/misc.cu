@@ -111,14 +111,14 @@ void reduce_to_column(Matrix* V, const Matrix* M) {
         return;
     }
     DevBuf<uint32_t> f(m);
-    DevBuf<off_t64> rp(size_t(m) + 1);
+    DevBuf<off_t64> rp(size_t(m) + 1, kMat);
     reduce_flags_kernel<<<grid_for(m, 256), 256, 0, ctx().stream>>>(M->rowptr, m, f.p);
     count_launch();
     check_launch("reduce_flags_kernel");
     exclusive_scan_u32(f.p, rp.p, m);
     uint64_t nnz;
     read_words(rp.p + m, &nnz, 1);
-    DevBuf<idx_t> ci(nnz);
+    DevBuf<idx_t> ci(nnz, kMat);
     memset_async(ci.p, 0, nnz * sizeof(idx_t));  // the single column index 0
     size_t rc = rp.n, cc = ci.n;
     matrix_replace(V, rp.detach(), rc, ci.detach(), cc, nnz);
@@ -135,14 +135,14 @@ void submatrix(Matrix* R, const Matrix* M, idx_t i0, idx_t j0, idx_t nr, idx_t n
     }
     DevBuf<uint32_t> cnt(nr);
     DevBuf<uint64_t> beg(nr);
-    DevBuf<off_t64> rp(size_t(nr) + 1);
+    DevBuf<off_t64> rp(size_t(nr) + 1, kMat);
     sub_count_kernel<<<grid_for(nr, 256), 256, 0, ctx().stream>>>(view(M), i0, j0, nr, nc, cnt.p, beg.p);
     count_launch();
     check_launch("sub_count_kernel");
     exclusive_scan_u32(cnt.p, rp.p, nr);
     uint64_t nnz;
     read_words(rp.p + nr, &nnz, 1);
-    DevBuf<idx_t> ci(nnz);
+    DevBuf<idx_t> ci(nnz, kMat);
     if (nnz) {
         sub_copy_kernel<<<grid_for(uint64_t(nr) * 32, 256), 256, 0, ctx().stream>>>(M->colidx, beg.p, rp.p, nr, j0, ci.p);
         count_launch();

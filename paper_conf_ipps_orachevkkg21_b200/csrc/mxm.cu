@@ -88,6 +88,7 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
         matrix_set_empty(C);
         return;
     }
+    trace_mark("mxm start");
     DevBuf<uint64_t> ub(m);
     DevBuf<uint2> range(m);
     DevBuf<uint4> desc(A->nnz);
@@ -119,6 +120,7 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     matrix_replace(C, tmp.rowptr, tmp.rowptr_cap, tmp.colidx, tmp.colidx_cap, tmp.nnz);
     tmp.rowptr = nullptr;
     tmp.colidx = nullptr;
+    trace_mark("mxm done");
 }
 
 void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {

@@ -815,6 +815,165 @@ __global__ void compact_kernel(const idx_t* __restrict__ scratch, const uint64_t
     }
 }
 
+// In-place compaction: the rows sit in one buffer at their capacity offsets
+// soff[r] >= rowptr[r]; move every row down to rowptr[r] without a second
+// buffer.  Destination tiles of kCT elements are claimed in increasing order
+// (atomic ticket).  A tile first loads its elements into registers and
+// publishes "read done"; it may then overwrite [d0, d1) once every earlier
+// tile that reads sources inside [d0, d1) has published.  Sources of
+// destination d lie at d + slack(row(d)), slack = soff - rowptr nondecreasing,
+// so those tiles are the ones in [t - 1 - slack(r0) / kCT, t).  Waits only
+// point at lower tickets, held by running blocks that never wait before
+// publishing, so the chain cannot deadlock.  Tiles with zero slack are
+// already in place and only publish.
+constexpr int kCThreads = 256, kCItems = 32;
+constexpr uint32_t kCT = kCThreads * kCItems;  // 8192 elements per tile
+constexpr uint32_t kCStage = 1024;             // rows of a tile staged in smem
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// index of the row holding position d: largest r in [lo, hi] with rp[r] <= d
+__device__ __forceinline__ uint32_t row_of(const uint64_t* rp, uint32_t lo, uint32_t hi, uint64_t d) {
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (rp[mid] <= d) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+// tile_row[t] = row holding position t*kCT (t < ntiles), tile_row[ntiles] =
+// nrows-1; src_lo[t] = source position of the tile's first element.
+__global__ void tile_rows_kernel(const uint64_t* __restrict__ rowptr, const uint64_t* __restrict__ soff,
+                                 idx_t nrows, uint64_t ntiles, uint32_t* __restrict__ tile_row,
+                                 uint64_t* __restrict__ src_lo) {
+    for (size_t r = blockIdx.x * size_t(blockDim.x) + threadIdx.x; r < nrows; r += size_t(gridDim.x) * blockDim.x) {
+        const uint64_t b = rowptr[r], e = rowptr[r + 1];
+        for (uint64_t t = (b + kCT - 1) / kCT; t * kCT < e; ++t) {
+            tile_row[t] = uint32_t(r);
+            src_lo[t] = t * kCT + (soff[r] - b);
+        }
+        if (r == nrows - 1) tile_row[ntiles] = uint32_t(r);
+    }
+}
+
+// Tiles that tile t must wait for: the j < t whose sources overlap [d0, d1).
+// src is strictly increasing in the destination, so tile j's sources lie in
+// [src_lo[j], src_lo[j+1]).  Overlap needs src_lo[j+1] > d0 and
+// src_lo[j] < d1: j in [J0 - 1, J1) with J0 the first tile whose src_lo
+// exceeds d0 and J1 the first whose src_lo reaches d1 (usually 1-2 tiles).
+__global__ void tile_deps_kernel(const uint64_t* __restrict__ src_lo, uint64_t ntiles, uint64_t nnz,
+                                 uint2* __restrict__ wait_range) {
+    for (size_t t = blockIdx.x * size_t(blockDim.x) + threadIdx.x; t < ntiles; t += size_t(gridDim.x) * blockDim.x) {
+        const uint64_t d0 = t * kCT, d1 = min(d0 + kCT, nnz);
+        // src_lo[j] <= j*kCT + slack(t) for j <= t: the answers lie within `back` tiles
+        const uint64_t back = (src_lo[t] - d0) / kCT + 2;
+        const uint64_t start = t > back ? t - back : 0;
+        auto first_above = [&](uint64_t x, bool strict) {  // first j in [start, t] with src_lo[j] > x (>= x)
+            uint64_t lo = start, hi = t;
+            while (lo < hi) {
+                const uint64_t mid = (lo + hi) >> 1;
+                const uint64_t v = src_lo[mid];
+                if (strict ? v <= x : v < x) lo = mid + 1; else hi = mid;
+            }
+            return lo;
+        };
+        const uint64_t j0 = first_above(d0, true);
+        const uint64_t j1 = first_above(d1, false);
+        wait_range[t] = make_uint2(uint32_t(j0 > 0 ? j0 - 1 : 0), uint32_t(min(j1, uint64_t(t))));
+    }
+}
+
+__global__ void __launch_bounds__(kCThreads)
+compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint64_t* __restrict__ rowptr,
+                       const uint32_t* __restrict__ tile_row, const uint2* __restrict__ wait_range,
+                       idx_t nrows, uint64_t nnz, uint32_t* flags, uint32_t* ticket) {
+    __shared__ uint64_t s_rp[kCStage + 1], s_sl[kCStage];
+    __shared__ uint32_t s_t, s_r0, s_r1;
+    __shared__ uint2 s_w;
+    const uint64_t ntiles = (nnz + kCT - 1) / kCT;
+    for (;;) {
+        if (threadIdx.x == 0) {
+            const uint32_t t = atomicAdd(ticket, 1u);
+            s_t = t;
+            if (t < ntiles) {
+                // rows holding d0 and (a bound on the row holding) d1-1
+                s_r0 = tile_row[t];
+                s_r1 = tile_row[t + 1];
+                s_w = wait_range[t];
+            }
+        }
+        __syncthreads();
+        const uint32_t t = s_t;
+        if (t >= ntiles) break;
+        const uint64_t d0 = uint64_t(t) * kCT, d1 = min(d0 + kCT, nnz);
+        const uint32_t r0 = s_r0, r1 = s_r1;
+        const uint64_t slack1 = soff[r1] - rowptr[r1];
+        if (slack1 == 0) {  // whole tile already in place (slack is nondecreasing)
+            if (threadIdx.x == 0) st_release_u32(&flags[t], 1u);
+            __syncthreads();
+            continue;
+        }
+        const uint32_t nr = r1 - r0 + 1;
+        const bool staged = nr <= kCStage;
+        if (staged) {
+            for (uint32_t i = threadIdx.x; i < nr; i += kCThreads) {
+                const uint64_t rp = rowptr[r0 + i];
+                s_rp[i] = rp;
+                s_sl[i] = soff[r0 + i] - rp;
+            }
+        }
+        __syncthreads();
+        idx_t v[kCItems];
+        uint32_t ri = 0;  // staged: row index relative to r0, advanced monotonically
+#pragma unroll
+        for (int k = 0; k < kCItems; ++k) {
+            const uint64_t d = d0 + uint32_t(k) * kCThreads + threadIdx.x;
+            if (d < d1) {
+                uint64_t src;
+                if (staged) {
+                    if (ri + 1 < nr && s_rp[ri + 1] <= d) {  // next row(s): binary search in smem
+                        uint32_t lo = ri + 1, hi = nr - 1;
+                        while (lo < hi) {
+                            const uint32_t mid = (lo + hi + 1) >> 1;
+                            if (s_rp[mid] <= d) lo = mid; else hi = mid - 1;
+                        }
+                        ri = lo;
+                    }
+                    src = d + s_sl[ri];
+                } else {
+                    const uint32_t r = row_of(rowptr, r0, r1, d);
+                    src = d + (soff[r] - rowptr[r]);
+                }
+                v[k] = buf[src];
+            }
+        }
+        // publish "read done": the barrier orders every thread's loads before
+        // thread 0's gpu-scope fence and release store
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            st_release_u32(&flags[t], 1u);
+        }
+        // wait for the earlier tiles that read sources inside [d0, d1)
+        for (uint32_t j = s_w.x + threadIdx.x; j < s_w.y; j += kCThreads)
+            while (ld_acquire_u32(&flags[j]) == 0) __nanosleep(64);
+        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < kCItems; ++k) {
+            const uint64_t d = d0 + uint32_t(k) * kCThreads + threadIdx.x;
+            if (d < d1) buf[d] = v[k];
+        }
+        __syncthreads();  // s_rp / s_t reuse
+    }
+}
+
 }  // namespace
 
 // ------------------------------------------------------------------------------
@@ -870,6 +1029,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
         return;
     }
     ensure_attrs();
+    trace_mark("engine start");
     // 1-3. bins
     DevBuf<uint64_t> cap(size_t(nrows) + 1);
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
@@ -899,8 +1059,11 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     const uint64_t scratch_total = h[0];
     cap.release();
     bin.release();
-    DevBuf<idx_t> scratch(scratch_total);
+    trace_mark("binning");
+    // the scratch is matrix storage: compacted in place it becomes colidx
+    DevBuf<idx_t> scratch(scratch_total, kMat);
     DevBuf<idx_t> ovf_rows(nrows);
+    trace_mark("scratch alloc");
 
     // 4. per-bin kernels, heaviest first, back to back on the library stream
     //    (persistent grids sized to the SM count x residency; rows are handed
@@ -936,13 +1099,38 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     ktime_end(t);
     count_launch(5);
     check_launch("warp_bin_kernel");
+    trace_mark("bin kernels");
     // 5. row offsets
-    DevBuf<off_t64> rowptr(size_t(nrows) + 1);
+    DevBuf<off_t64> rowptr(size_t(nrows) + 1, kMat);
     exclusive_scan_u32(counts.p, rowptr.p, nrows);
     read_words(rowptr.p + nrows, h, 1);
     const uint64_t nnz = h[0];
-    DevBuf<idx_t> colidx(nnz);
-    if (nnz) {
+    ovf_rows.release();
+    counts.release();
+    // 6. compaction: in place when the capacity slack is small (the result
+    //    keeps the buffer, colidx_cap >= nnz), else into an exact buffer
+    const bool inplace = scratch_total - nnz <= scratch_total / 8;
+    DevBuf<idx_t> colidx;
+    if (nnz && inplace) {
+        const uint64_t ntiles = ceil_div(nnz, kCT);
+        // flags[ntiles] | ticket | tile_row[ntiles + 1]; src_lo[ntiles]; wait_range[ntiles]
+        DevBuf<uint32_t> flags(2 * ntiles + 2);
+        DevBuf<uint64_t> src_lo(ntiles);
+        DevBuf<uint2> wait_range(ntiles);
+        uint32_t* tile_row = flags.p + ntiles + 1;
+        memset_async(flags.p, 0, (ntiles + 1) * sizeof(uint32_t));
+        t = ktime_begin("compact", st);
+        tile_rows_kernel<<<gb, 256, 0, st>>>(rowptr.p, soff.p, nrows, ntiles, tile_row, src_lo.p);
+        tile_deps_kernel<<<(unsigned)std::min<uint64_t>(ceil_div(ntiles, 256), uint64_t(nsm) * 8), 256, 0, st>>>(
+            src_lo.p, ntiles, nnz, wait_range.p);
+        compact_inplace_kernel<<<nsm * 8, kCThreads, 0, st>>>(scratch.p, soff.p, rowptr.p, tile_row, wait_range.p,
+                                                             nrows, nnz, flags.p, flags.p + ntiles);
+        count_launch(2);
+        ktime_end(t);
+        count_launch();
+        check_launch("compact_inplace_kernel");
+    } else if (nnz) {
+        colidx.alloc(nnz, kMat);
         const unsigned gc = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(nrows) * 32, 256), uint64_t(nsm) * 16);
         t = ktime_begin("compact", st);
         compact_kernel<<<gc, 256, 0, st>>>(scratch.p, soff.p, rowptr.p, nrows, colidx.p);
@@ -950,8 +1138,15 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
         count_launch();
         check_launch("compact_kernel");
     }
-    size_t rcap = rowptr.n, ccap = colidx.n;
-    matrix_replace(out, rowptr.detach(), rcap, colidx.detach(), ccap, nnz);
+    trace_mark("compact");
+    size_t rcap = rowptr.n;
+    if (nnz && inplace) {
+        size_t ccap = scratch.n;
+        matrix_replace(out, rowptr.detach(), rcap, scratch.detach(), ccap, nnz);
+    } else {
+        size_t ccap = colidx.n;
+        matrix_replace(out, rowptr.detach(), rcap, colidx.detach(), ccap, nnz);
+    }
 }
 
 void engine_thresholds(uint64_t* out, uint32_t* n) {

@@ -37,6 +37,26 @@ def test_build_heavy_rows(sp):
     assert_same(M, O, "build heavy")
 
 
+@pytest.mark.parametrize("nrows,per_row,ncols,dup_every", [(1 << 20, 4, 1 << 20, 16), (1 << 12, 3000, 1 << 22, 5),
+                                                            (1 << 16, 40, 1 << 16, 1)])
+def test_build_inplace_compaction(sp, nrows, per_row, ncols, dup_every):
+    """Row-engine compaction regimes: a few duplicates per many rows leave a
+    small capacity slack (in-place ordered compaction over ~500-1500 tiles of
+    8192 entries; short rows take the unstaged row search, long rows the
+    smem-staged one); dup_every=1 gives a large slack (out-of-place path)."""
+    rng = np.random.default_rng(nrows + per_row)
+    r = np.repeat(np.arange(nrows, dtype=np.uint32), per_row)
+    c = rng.integers(0, ncols, len(r)).astype(np.uint32)
+    c2 = c.reshape(nrows, per_row)
+    dup_rows = np.arange(0, nrows, dup_every)
+    c2[dup_rows, 1] = c2[dup_rows, 0]  # one forced duplicate in every dup_every-th row
+    if dup_every == 1:
+        c2[:, per_row // 2:] = c2[:, :per_row - per_row // 2]
+    perm = rng.permutation(len(r))
+    M, O = both_from_pairs(sp, nrows, ncols, r[perm], c[perm])
+    assert_same(M, O, "build in-place compaction")
+
+
 def test_build_empty_and_errors(sp):
     M = sp.Matrix.new(10, 10)
     M.build(np.zeros(0, np.uint32), np.zeros(0, np.uint32))
