@@ -72,7 +72,6 @@ enum {
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 512
 // hash bins: ub limits (each sized so its tables fit the residency below)
 constexpr uint64_t kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480, kH6 = 40960;
-constexpr uint32_t kMaxProbe = 96;
 constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
@@ -192,16 +191,16 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
     return uint32_t(tot);
 }
 
-// Call f(c) for every product of row r.  Warps take chunks of 32*U
-// consecutive products; per 32-product step a lane loads one candidate
-// segment (32 consecutive segments cover 32 consecutive products), a 5-step
-// shuffle search finds each lane's segment, and the U loads of a chunk
-// are issued before any insert.  Ends with a barrier.
+// Call f(c) for every product of row r.  Thread t takes U consecutive
+// products q0 = (t + i*THREADS)*U .. q0+U-1 of the concatenated segments:
+// one binary search over the staged segment ends for q0, then a linear
+// advance (segments average tens of products, so a run rarely crosses more
+// than one boundary); the U loads are issued before any insert.  A warp
+// covers 32*U consecutive products, i.e. a few sectors of each B row.
+// Ends with a barrier.
 template <int THREADS, int U, typename F>
 __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, const idx_t** sd_ptr,
                                                uint32_t* sd_end, uint32_t batch, uint64_t* s_scan, F&& f) {
-    constexpr uint32_t NW = THREADS / 32, CH = 32 * U;
-    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t nseg = num_segs(s, r);
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
         uint32_t ns;
@@ -209,29 +208,27 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, cons
 #ifdef SPBLA_PROBE
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
-        for (uint32_t base = wib * CH; base < total; base += NW * CH) {
-            uint32_t lo = 0, hi = ns - 1;  // segment holding product `base`
+        for (uint32_t q0 = threadIdx.x * U; q0 < total; q0 += THREADS * U) {
+            uint32_t lo = 0, hi = ns - 1;  // first segment whose end exceeds q0
             while (lo < hi) {
                 const uint32_t mid = (lo + hi) >> 1;
-                if (sd_end[mid] <= base) lo = mid + 1; else hi = mid;
+                if (sd_end[mid] <= q0) lo = mid + 1; else hi = mid;
             }
-            uint32_t sb = lo;
+            uint32_t k = lo, end = sd_end[lo];
+            const idx_t* p = sd_ptr[lo];
             idx_t v[U];
 #pragma unroll
             for (int u = 0; u < U; ++u) {
-                const uint32_t qb = base + 32u * u, q = qb + lane;
-                const uint32_t cand = sb + lane;
-                const uint32_t E = cand < ns ? sd_end[cand] : 0xFFFFFFFFu;
-                const unsigned long long P = cand < ns ? (unsigned long long)sd_ptr[cand] : 0ull;
-                uint32_t pos = 0;
-#pragma unroll
-                for (int st = 16; st > 0; st >>= 1) {
-                    const uint32_t t = __shfl_sync(FULL, E, pos + st - 1);
-                    if (t <= q) pos += st;
+                const uint32_t q = q0 + u;
+                v[u] = kEmpty;
+                if (q < total) {
+                    while (q >= end) {  // staged segments are non-empty
+                        ++k;
+                        end = sd_end[k];
+                        p = sd_ptr[k];
+                    }
+                    v[u] = __ldg(p + q);
                 }
-                const idx_t* ps = (const idx_t*)__shfl_sync(FULL, P, pos > 31 ? 31 : pos);
-                v[u] = q < total ? __ldg(ps + q) : kEmpty;
-                sb += __popc(__ballot_sync(FULL, E <= qb + 32));
             }
 #pragma unroll
             for (int u = 0; u < U; ++u)
@@ -288,47 +285,6 @@ __device__ __forceinline__ uint32_t emit_bitmap(const uint32_t* bm, uint32_t nwo
     return total;
 }
 
-// Ordered emission of an order-preserving hash table: clusters (maximal runs
-// of occupied slots) are mutually ordered, so the element at slot i goes to
-// (#occupied slots before its cluster start cs) + (its rank in the cluster).
-template <int NW>
-__device__ __forceinline__ uint32_t emit_table_ranked(const idx_t* tab, uint32_t nslots, idx_t* __restrict__ out,
-                                                      uint32_t* s_w) {
-    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
-    const uint32_t chunk = ((nslots + NW - 1) / NW + 31) & ~31u;
-    const uint32_t b = wib * chunk, e = min(b + chunk, nslots);
-    uint32_t cnt = 0;
-    for (uint32_t i0 = b; i0 < e; i0 += 32) {
-        const uint32_t i = i0 + lane;
-        cnt += __popc(__ballot_sync(FULL, i < e && tab[i] != kEmpty));
-    }
-    if (lane == 0) s_w[wib] = cnt;
-    __syncthreads();
-    scan_warp_counts<NW>(s_w);
-    uint32_t pos = s_w[wib];
-    const uint32_t lt = (1u << lane) - 1u;
-    for (uint32_t i0 = b; i0 < e; i0 += 32) {
-        const uint32_t i = i0 + lane;
-        const idx_t v = i < e ? tab[i] : kEmpty;
-        const uint32_t m = __ballot_sync(FULL, v != kEmpty);
-        if (v != kEmpty) {
-            uint32_t cs = i;
-            while (cs > 0 && tab[cs - 1] != kEmpty) --cs;
-            uint32_t rank = 0;
-            for (uint32_t j = cs; j < nslots; ++j) {
-                const idx_t w = tab[j];
-                if (w == kEmpty) break;
-                rank += (w < v);
-            }
-            out[pos + __popc(m & lt) - (i - cs) + rank] = v;
-        }
-        pos += __popc(m);
-    }
-    const uint32_t total = s_w[32];
-    __syncthreads();
-    return total;
-}
-
 __device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, int threads) {
     // p is 16-byte aligned; vector stores for the bulk
     uint4* p4 = reinterpret_cast<uint4*>(p);
@@ -338,91 +294,55 @@ __device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, 
 }
 
 // ---- 4b. block hash / span-bitmap bins --------------------------------------
-// Bucketed ORDER-PRESERVING hash: bucket b = floor((c - lo) * nb / span) is
-// monotone in c, so buckets are mutually ordered.  Each bucket has 8 slots
-// (mean load 4) and a fill counter: an insert is one smem atomicAdd on the
-// counter and one store - no probing, no CAS, no lane divergence; duplicates
-// are dropped at emission.  Products arriving at a full bucket go to a small
-// monotone linear-probing overflow table (atomicCAS, duplicate-free).
-// Emission: per-thread runs of buckets; each bucket is sorted in registers by
-// an 8-input Batcher network, merged with its (rare) overflow elements and
-// deduplicated; a block scan of the per-thread unique counts gives the output
-// offsets (the sort is repeated in the write pass instead of keeping 8
-// registers per bucket live across the scan).
-__device__ __forceinline__ void cswap(idx_t& a, idx_t& b) {
-    const idx_t x = min(a, b), y = max(a, b);
+// Bucketed ORDER-PRESERVING hash: bucket b = floor((c - lo) / W) is monotone
+// in c, so buckets are mutually ordered.  Each bucket has 8 slots of 16-bit
+// offsets c - lo - b*W (W <= 65535; 0xFFFF marks an empty slot) and a fill
+// counter: an insert is one smem atomicAdd on the counter and one 16-bit
+// store - no probing, no CAS, no lane divergence; duplicates are dropped at
+// emission.  A product arriving at a full bucket is appended to a small
+// overflow list.  nb = ub/4 buckets (mean load <= 4, ~5 bytes of smem per
+// product).
+//
+// Emission, per thread a run of k buckets:
+//  pass A: two buckets at a time in 16x2 SIMD registers (VIMNMX.U16x2): an
+//          8-input Batcher network sorts both, the sorted slots are written
+//          back in place, the distinct values are counted (n_valid minus
+//          adjacent equal pairs, via max(x_i, x_{i-1}+1) - x_i in 16x2
+//          arithmetic).  A bucket that overflowed is listed instead;
+//  overflow: one warp per listed bucket gathers its 8 slots and its list
+//          entries (ballot over the list), bitonic-sorts <= 32 values across
+//          lanes, dedups, and parks the result in a side area;
+//  block scan of the per-thread distinct counts;
+//  pass B: stream each sorted bucket (or parked overflow bucket) to the row's
+//          output, skipping adjacent duplicates - no sort in this pass.
+__device__ __forceinline__ void cswap2(uint32_t& a, uint32_t& b) {
+    const uint32_t x = __vminu2(a, b), y = __vmaxu2(a, b);
     a = x;
     b = y;
 }
-__device__ __forceinline__ void sort8(idx_t (&v)[8]) {  // Batcher odd-even merge sort, 19 comparators
-    cswap(v[0], v[1]); cswap(v[2], v[3]); cswap(v[4], v[5]); cswap(v[6], v[7]);
-    cswap(v[0], v[2]); cswap(v[1], v[3]); cswap(v[4], v[6]); cswap(v[5], v[7]);
-    cswap(v[1], v[2]); cswap(v[5], v[6]);
-    cswap(v[0], v[4]); cswap(v[1], v[5]); cswap(v[2], v[6]); cswap(v[3], v[7]);
-    cswap(v[2], v[4]); cswap(v[3], v[5]);
-    cswap(v[1], v[2]); cswap(v[3], v[4]); cswap(v[5], v[6]);
+__device__ __forceinline__ void sort8x2(uint32_t (&v)[8]) {  // Batcher odd-even merge sort, 19 comparators
+    cswap2(v[0], v[1]); cswap2(v[2], v[3]); cswap2(v[4], v[5]); cswap2(v[6], v[7]);
+    cswap2(v[0], v[2]); cswap2(v[1], v[3]); cswap2(v[4], v[6]); cswap2(v[5], v[7]);
+    cswap2(v[1], v[2]); cswap2(v[5], v[6]);
+    cswap2(v[0], v[4]); cswap2(v[1], v[5]); cswap2(v[2], v[6]); cswap2(v[3], v[7]);
+    cswap2(v[2], v[4]); cswap2(v[3], v[5]);
+    cswap2(v[1], v[2]); cswap2(v[3], v[4]); cswap2(v[5], v[6]);
 }
-
-constexpr uint32_t kOvSlack = 128;
-
-// Sorted bucket b (kEmpty-padded) -> emit (or count when out == nullptr) its
-// distinct values merged with the sorted overflow run ovs[oi, oe).
-__device__ __forceinline__ uint32_t bucket_emit(const uint16_t* tab, const uint32_t* cnt, uint32_t b,
-                                                idx_t base, const idx_t* ovs, uint32_t oi, uint32_t oe,
-                                                idx_t* __restrict__ out) {
-    const uint32_t n = min(cnt[b], 8u);
-    const uint4 w = reinterpret_cast<const uint4*>(tab)[b];  // 8 x 16-bit offsets
-    const uint32_t q4[4] = {w.x, w.y, w.z, w.w};
-    idx_t v[8];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-        v[2 * i] = uint32_t(2 * i) < n ? base + (q4[i] & 0xFFFFu) : kEmpty;
-        v[2 * i + 1] = uint32_t(2 * i + 1) < n ? base + (q4[i] >> 16) : kEmpty;
-    }
-    sort8(v);
-    uint32_t m = 0;
-    idx_t prev = kEmpty;
-    if (oi == oe) {
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            if (v[j] != kEmpty && v[j] != prev) {
-                if (out) out[m] = v[j];
-                ++m;
-            }
-            prev = v[j];
-        }
-        return m;
-    }
-    // merge with the overflow run (both sorted), dropping duplicates
-    int j = 0;
-    uint32_t q = oi;
-    for (;;) {
-        const idx_t a = j < 8 ? v[j] : kEmpty;
-        const idx_t c = q < oe ? ovs[q] : kEmpty;
-        if (a == kEmpty && c == kEmpty) break;
-        idx_t t;
-        if (a <= c) {
-            t = a;
-            ++j;
-        } else {
-            t = c;
-            ++q;
-        }
-        if (t != prev) {
-            if (out) out[m] = t;
-            ++m;
-            prev = t;
-        }
-    }
-    return m;
+__device__ __forceinline__ uint32_t vadd2(uint32_t a, uint32_t b) {  // per-16-bit-lane add (wrapping)
+    uint32_t r;
+    asm("add.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+    return r;
 }
+constexpr uint32_t kOvfFlag = 0x80000000u;
 
-// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | tab[MAXB*8] u16 | cnt[MAXB] | ovt[OVS+kOvSlack] | ovs[OVS+kOvSlack]
-// Bucket b = floor((c - lo) / W) (W = ceil(span / nb) <= 65535, computed with
-// an exact 48-bit reciprocal), each slot the 16-bit offset c - lo - b*W:
-// 20 bytes per bucket of mean load 4, so ~5 bytes of smem per product.
-// (ovs holds the sorted overflow elements: at most the table's OVS+kOvSlack slots)
-template <int THREADS, uint32_t MAXB, uint32_t OVS, uint32_t BATCH, int MINB, int FLATU>
+template <int E>
+__device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]);
+
+// dynamic smem: tab[MAXB] uint4 | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | ovl[OVCAP] |
+//               pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | s_cnt[THREADS]
+// (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
+// which are dead once the products are inserted: BATCH * 3 >= THREADS)
+template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU>
 __global__ void __launch_bounds__(THREADS, MINB)
 hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
                 const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
@@ -430,16 +350,23 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
     constexpr int NW = THREADS / 32;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
-    uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
-    uint16_t* tab = reinterpret_cast<uint16_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
-    uint32_t* bmw = reinterpret_cast<uint32_t*>(tab);  // bitmap-mode view: MAXB * 5 words
-    uint32_t* bcnt = reinterpret_cast<uint32_t*>(tab + MAXB * 8);
-    idx_t* ovt = bcnt + MAXB;
-    idx_t* ovs = ovt + OVS + kOvSlack;
+    uint4* tab4 = reinterpret_cast<uint4*>(smem_raw);
+    uint16_t* tab16 = reinterpret_cast<uint16_t*>(smem_raw);
+    uint32_t* bmw = reinterpret_cast<uint32_t*>(smem_raw);  // bitmap-mode view: MAXB * 5 words
+    uint32_t* bcnt = reinterpret_cast<uint32_t*>(smem_raw + MAXB * sizeof(uint4));
+    const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(bcnt + MAXB);
+    uint32_t* sd_end = reinterpret_cast<uint32_t*>(sd_ptr + BATCH);
+    idx_t* ovl = sd_end + BATCH;
+    uint16_t* pool = reinterpret_cast<uint16_t*>(ovl + OVCAP);
+    uint32_t* obl = reinterpret_cast<uint32_t*>(pool + OVCAP);  // OVCAP even
+    uint32_t* obcnt = obl + OBCAP;
+    uint32_t* s_cnt = obcnt + OBCAP;
+    uint32_t* wbuf = reinterpret_cast<uint32_t*>(sd_ptr);
+    static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0, "hash bin layout");
     __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_item, s_flag, s_novf;
+    __shared__ uint32_t s_item, s_flag, s_novf, s_nob, s_pool;
+    const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
     PROBE_DECL
     for (;;) {
@@ -447,6 +374,8 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             s_item = lo_i + atomicAdd(work, 1u);
             s_flag = 0;
             s_novf = 0;
+            s_nob = 0;
+            s_pool = 0;
         }
         __syncthreads();
         const uint32_t item = s_item;
@@ -487,81 +416,160 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         }
         const uint32_t W = uint32_t((span + nb - 1) / nb);
         const uint64_t M16 = ((((uint64_t(1) << 48) + W - 1) / W) << 16);  // ceil(2^48 / W) << 16
-        const uint32_t ovn = min(max(u / 16, 64u), OVS);
-        const uint32_t ovslots = ovn + kOvSlack;
+        fill_words(reinterpret_cast<uint32_t*>(tab4), nb * 4, 0xFFFFFFFFu, THREADS);
         fill_words(bcnt, nb, 0u, THREADS);
-        fill_words(ovt, ovslots, kEmpty, THREADS);
         __syncthreads();
         PROBE(2);
-        const uint64_t oscale = (uint64_t(ovn) << 32) / span;
         block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
             const uint64_t d = uint64_t(c - clo);
             const uint32_t b = uint32_t(__umul64hi(d, M16));  // floor(d / W), exact for W < 2^16
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
             if (slot < 8) {
-                tab[b * 8 + slot] = uint16_t(uint32_t(d) - b * W);
-                return;
-            }
-            // bucket full: overflow table (monotone linear probing, no wrap)
-            uint32_t h = uint32_t((d * oscale) >> 32);
-            for (uint32_t probe = 0;; ++probe) {
-                const idx_t cur = ovt[h];
-                if (cur == c) return;
-                if (cur == kEmpty) {
-                    const idx_t old = atomicCAS(&ovt[h], kEmpty, c);
-                    if (old == kEmpty) {
-                        atomicAdd(&s_novf, 1u);
-                        return;
-                    }
-                    if (old == c) return;
-                }
-                if (++h >= ovslots || probe >= kMaxProbe) {
-                    s_flag = 1;  // hand the row to the bitmap bin
-                    return;
-                }
+                tab16[b * 8 + slot] = uint16_t(uint32_t(d) - b * W);
+            } else {
+                const uint32_t i = atomicAdd(&s_novf, 1u);
+                if (i < OVCAP) ovl[i] = c; else s_flag = 1;
             }
         });
-        if (s_flag) {
+        if (s_flag) {  // overflow list full: hand the row to the bitmap bin
             if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
             __syncthreads();  // everyone has read s_flag / s_item before reuse
             continue;
         }
         PROBE(4);
-        const uint32_t novf = s_novf;
-        if (novf) emit_table_ranked<NW>(ovt, ovslots, ovs, s_w);  // sorted overflow -> ovs (smem)
-        // thread t owns buckets [t*k, (t+1)*k); ovs runs located by bucket
-        const uint32_t k = (nb + THREADS - 1) / THREADS;
-        const uint32_t b0 = threadIdx.x * k, b1 = min(b0 + k, nb);
-        auto obucket = [&](uint32_t i) { return uint32_t(__umul64hi(uint64_t(ovs[i] - clo), M16)); };
-        uint32_t o0 = 0;
-        if (novf) {
-            uint32_t lo = 0, hi = novf;
-            while (lo < hi) {
-                const uint32_t mid = (lo + hi) >> 1;
-                if (obucket(mid) < b0) lo = mid + 1; else hi = mid;
+        // ---- pass A: sort pairs of buckets in 16x2 SIMD, count distinct values
+        const uint32_t k = 2 * ((nb + 2 * THREADS - 1) / (2 * THREADS));
+        const uint32_t b0 = min(threadIdx.x * k, nb), b1 = min(b0 + k, nb);
+        uint32_t cnt = 0;
+        for (uint32_t b = b0; b < b1; b += 2) {
+            const bool two = b + 1 < b1;
+            const uint32_t n0 = bcnt[b], n1 = two ? bcnt[b + 1] : 0u;
+            uint4 w0 = tab4[b];
+            uint4 w1 = two ? tab4[b + 1] : make_uint4(~0u, ~0u, ~0u, ~0u);
+            if (n0 > 8 || n1 > 8) {  // rare: list the overflowing bucket(s), sort the rest
+                if (n0 > 8) {
+                    const uint32_t j = atomicAdd(&s_nob, 1u);
+                    if (j < OBCAP) obl[j] = b; else s_flag = 1;
+                    bcnt[b] = kOvfFlag | j;
+                    w0 = make_uint4(~0u, ~0u, ~0u, ~0u);
+                }
+                if (n1 > 8) {
+                    const uint32_t j = atomicAdd(&s_nob, 1u);
+                    if (j < OBCAP) obl[j] = b + 1; else s_flag = 1;
+                    bcnt[b + 1] = kOvfFlag | j;
+                    w1 = make_uint4(~0u, ~0u, ~0u, ~0u);
+                }
             }
-            o0 = lo;
+            // x[i] = (slot i of bucket b+1) << 16 | (slot i of bucket b)
+            uint32_t x[8];
+            x[0] = __byte_perm(w0.x, w1.x, 0x5410); x[1] = __byte_perm(w0.x, w1.x, 0x7632);
+            x[2] = __byte_perm(w0.y, w1.y, 0x5410); x[3] = __byte_perm(w0.y, w1.y, 0x7632);
+            x[4] = __byte_perm(w0.z, w1.z, 0x5410); x[5] = __byte_perm(w0.z, w1.z, 0x7632);
+            x[6] = __byte_perm(w0.w, w1.w, 0x5410); x[7] = __byte_perm(w0.w, w1.w, 0x7632);
+            sort8x2(x);
+            // adjacent equal pairs: max(x_i, x_{i-1} + 1) - x_i is 1 iff x_i == x_{i-1}
+            // (an empty 0xFFFF predecessor wraps to 0 and counts nothing)
+            uint32_t smax = 0, sx = 0;
+#pragma unroll
+            for (int i = 1; i < 8; ++i) {
+                smax = vadd2(smax, __vmaxu2(x[i], vadd2(x[i - 1], 0x00010001u)));
+                sx = vadd2(sx, x[i]);
+            }
+            const uint32_t d2 = vadd2(smax, vadd2(~sx, 0x00010001u));  // smax - sx per 16-bit lane
+            const uint32_t v0 = n0 > 8 ? 0u : n0, v1 = n1 > 8 ? 0u : n1;
+            cnt += v0 - (d2 & 0xFFFFu) + v1 - (d2 >> 16);
+            uint4 s0, s1;
+            s0.x = __byte_perm(x[0], x[1], 0x5410); s1.x = __byte_perm(x[0], x[1], 0x7632);
+            s0.y = __byte_perm(x[2], x[3], 0x5410); s1.y = __byte_perm(x[2], x[3], 0x7632);
+            s0.z = __byte_perm(x[4], x[5], 0x5410); s1.z = __byte_perm(x[4], x[5], 0x7632);
+            s0.w = __byte_perm(x[6], x[7], 0x5410); s1.w = __byte_perm(x[6], x[7], 0x7632);
+            if (n0 <= 8) tab4[b] = s0;
+            if (two && n1 <= 8) tab4[b + 1] = s1;
         }
-        uint64_t cnt = 0;
-        uint32_t oi = o0;
-        for (uint32_t b = b0; b < b1; ++b) {
-            uint32_t oe = oi;
-            if (bcnt[b] > 8)
-                while (oe < novf && obucket(oe) == b) ++oe;
-            cnt += bucket_emit(tab, bcnt, b, clo + b * W, ovs, oi, oe, nullptr);
-            oi = oe;
+        s_cnt[threadIdx.x] = cnt;
+        __syncthreads();
+        const uint32_t nob = s_nob;
+        if (s_flag) {
+            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            __syncthreads();
+            continue;
+        }
+        if (nob) {
+            // ---- overflow buckets: one warp each, <= 32 values sorted across lanes
+            const uint32_t novf = s_novf;
+            uint32_t* wb = wbuf + wib * 32;
+            const uint32_t lt = (1u << lane) - 1u;
+            for (uint32_t j = wib; j < nob; j += NW) {
+                const uint32_t b = obl[j];
+                const idx_t base = clo + b * W;
+                uint32_t filled = 8;
+                for (uint32_t i0 = 0; i0 < novf; i0 += 32) {
+                    const uint32_t i = i0 + lane;
+                    const idx_t c = i < novf ? ovl[i] : kEmpty;
+                    const bool match = c != kEmpty && uint32_t(__umul64hi(uint64_t(c - clo), M16)) == b;
+                    const uint32_t m = __ballot_sync(FULL, match);
+                    const uint32_t rank = filled + __popc(m & lt);
+                    if (match && rank < 32) wb[rank] = c;
+                    filled += __popc(m);
+                }
+                __syncwarp();
+                if (filled > 32) {  // warp-uniform
+                    if (lane == 0) s_flag = 1;
+                    continue;
+                }
+                idx_t xv[1];
+                xv[0] = lane < 8 ? base + tab16[b * 8 + lane] : (lane < filled ? wb[lane] : kEmpty);
+                __syncwarp();
+                warp_bitonic_sort<1>(xv);
+                const idx_t prev = __shfl_up_sync(FULL, xv[0], 1);
+                const bool uniq = xv[0] != kEmpty && (lane == 0 || xv[0] != prev);
+                const uint32_t um = __ballot_sync(FULL, uniq);
+                const uint32_t m = __popc(um), rank = __popc(um & lt);
+                // the first 8 distinct values go back to the bucket's slots
+                // (0xFFFF-padded), the rest to the pool (extras <= list entries)
+                const uint32_t extras = m > 8 ? m - 8 : 0u;
+                uint32_t off = 0;
+                if (lane == 0 && extras) off = atomicAdd(&s_pool, extras);
+                off = __shfl_sync(FULL, off, 0);
+                if (uniq) {
+                    const uint16_t o = uint16_t(xv[0] - base);
+                    if (rank < 8) tab16[b * 8 + rank] = o; else pool[off + rank - 8] = o;
+                }
+                if (lane < 8 && lane >= m) tab16[b * 8 + lane] = 0xFFFFu;
+                if (lane == 0) {
+                    obcnt[j] = (extras << 16) | off;
+                    atomicAdd(&s_cnt[b / k], m);
+                }
+            }
+            __syncthreads();
+            if (s_flag) {
+                if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+                __syncthreads();
+                continue;
+            }
         }
         PROBE(5);
         uint64_t total;
-        uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(cnt, s_scan, &total));
+        uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(s_cnt[threadIdx.x], s_scan, &total));
         PROBE(6);
-        oi = o0;
+        // ---- pass B: stream the sorted buckets, skipping adjacent duplicates
         for (uint32_t b = b0; b < b1; ++b) {
-            uint32_t oe = oi;
-            if (bcnt[b] > 8)
-                while (oe < novf && obucket(oe) == b) ++oe;
-            pos += bucket_emit(tab, bcnt, b, clo + b * W, ovs, oi, oe, out + pos);
-            oi = oe;
+            const uint32_t n = bcnt[b];
+            const idx_t base = clo + b * W;
+            const uint4 w = tab4[b];
+            const uint32_t q[4] = {w.x, w.y, w.z, w.w};
+            uint32_t prev = 0xFFFFu;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const uint32_t v = (q[i >> 1] >> ((i & 1) * 16)) & 0xFFFFu;
+                if (v != 0xFFFFu && v != prev) out[pos++] = base + v;
+                prev = v;
+            }
+            if (n & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
+                const uint32_t e = obcnt[n & ~kOvfFlag], m = e >> 16, off = e & 0xFFFFu;
+                for (uint32_t i = 0; i < m; ++i) out[pos + i] = base + pool[off + i];
+                pos += m;
+            }
         }
         if (threadIdx.x == 0) counts[r] = uint32_t(total);
         __syncthreads();
@@ -982,22 +990,26 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // batch, blocks per SM, loads in flight>; smem per block is checked against
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
 constexpr uint32_t kDBatch = 2048;
-constexpr size_t hash_smem(uint32_t batch, uint32_t buckets, uint32_t ovs) {
-    return batch * kSegBytes + buckets * (8 * sizeof(uint16_t) + sizeof(uint32_t)) + 2 * (ovs + kOvSlack) * sizeof(idx_t);
+constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, uint32_t ovcap, uint32_t obcap) {
+    return buckets * (sizeof(uint4) + sizeof(uint32_t)) + batch * kSegBytes + ovcap * (sizeof(idx_t) + sizeof(uint16_t)) +
+           obcap * 2 * sizeof(uint32_t) + threads * sizeof(uint32_t);
 }
-#define HBIN(NAME, T, UB, OVS, BATCH, PERSM, U)                                                    \
+#define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U)                                           \
     constexpr int NAME##_T = T, NAME##_PERSM = PERSM, NAME##_U = U;                                \
-    constexpr uint32_t NAME##_B = uint32_t(UB / 4), NAME##_OVS = OVS, NAME##_BATCH = BATCH;        \
-    constexpr size_t NAME##_SMEM = hash_smem(BATCH, uint32_t(UB / 4), OVS);                      \
+    constexpr uint32_t NAME##_B = uint32_t(UB / 4), NAME##_OVCAP = OVCAP, NAME##_OBCAP = OBCAP,     \
+                       NAME##_BATCH = BATCH;                                                       \
+    constexpr size_t NAME##_SMEM = hash_smem(T, BATCH, uint32_t(UB / 4), OVCAP, OBCAP);            \
     static_assert(PERSM * (NAME##_SMEM + 1024 + 600) <= 228 * 1024, #NAME " residency");          \
     static_assert(PERSM * T <= 2048, #NAME " threads");
-HBIN(H1, 128, kH1, 64, 256, 12, 4)
-HBIN(H2, 128, kH2, 128, 256, 12, 4)
-HBIN(H3, 256, kH3, 256, 384, 6, 4)
-HBIN(H4, 256, kH4, 512, 256, 4, 4)
-HBIN(H5, 512, kH5, 512, 256, 2, 8)
-HBIN(H6, 1024, kH6, 1024, 256, 1, 8)
-#define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVS, N##_BATCH, N##_PERSM, N##_U>
+// <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread>
+// (expected per row at mean load 4: list ~ub/130, buckets ~ub/190)
+HBIN(H1, 128, kH1, 64, 16, 256, 12, 4)
+HBIN(H2, 128, kH2, 64, 32, 256, 12, 4)
+HBIN(H3, 256, kH3, 128, 64, 384, 6, 4)
+HBIN(H4, 256, kH4, 256, 128, 256, 4, 8)
+HBIN(H5, 512, kH5, 384, 256, 256, 2, 8)
+HBIN(H6, 1024, kH6, 768, 512, 384, 1, 8)
+#define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U>
 #define HASH1 HASHK(H1)
 #define HASH2 HASHK(H2)
 #define HASH3 HASHK(H3)
