@@ -295,51 +295,69 @@ __device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, 
 
 // ---- 4b. block hash / span-bitmap bins --------------------------------------
 // Bucketed ORDER-PRESERVING hash: bucket b = floor((c - lo) / W) is monotone
-// in c, so buckets are mutually ordered.  Each bucket has 8 slots of 16-bit
+// in c, so buckets are mutually ordered.  A bucket has 16 slots of 16-bit
 // offsets c - lo - b*W (W <= 65535; 0xFFFF marks an empty slot) and a fill
 // counter: an insert is one smem atomicAdd on the counter and one 16-bit
 // store - no probing, no CAS, no lane divergence; duplicates are dropped at
-// emission.  A product arriving at a full bucket is appended to a small
-// overflow list.  nb = ub/4 buckets (mean load <= 4, ~5 bytes of smem per
-// product).
+// emission.  nb = ub/8 buckets (mean load <= 8, 4.5 bytes of smem per
+// product); a product arriving at a full bucket (p ~ 0.4%) is appended to a
+// small overflow list.  The table is stored word-transposed: word w (slots
+// 2w, 2w+1) of bucket b at tabw[w*MAXB + b], so a warp reading 32 adjacent
+// buckets touches 32 banks.
 //
-// Emission, per thread a run of k buckets:
-//  pass A: two buckets at a time in 16x2 SIMD registers (VIMNMX.U16x2): an
-//          8-input Batcher network sorts both, the sorted slots are written
-//          back in place, the distinct values are counted (n_valid minus
-//          adjacent equal pairs, via max(x_i, x_{i-1}+1) - x_i in 16x2
-//          arithmetic).  A bucket that overflowed is listed instead;
-//  overflow: one warp per listed bucket gathers its 8 slots and its list
+// Emission: thread t owns buckets t, t+T, t+2T, ... (k <= KMAX of them).
+//  pass A: two buckets at a time in 16x2 SIMD registers (VIMNMX.U16x2): a
+//          16-input Batcher network (63 comparators) sorts both, the sorted
+//          slots are written back, the distinct values are counted (n_valid
+//          minus adjacent equal pairs, via max(x_i, x_{i-1}+1) - x_i summed
+//          in 32-bit arithmetic).  A bucket that overflowed is listed instead;
+//  overflow: one warp per listed bucket gathers its 16 slots and its list
 //          entries (ballot over the list), bitonic-sorts <= 32 values across
-//          lanes, dedups, and parks the result in a side area;
-//  block scan of the per-thread distinct counts;
-//  pass B: stream each sorted bucket (or parked overflow bucket) to the row's
-//          output, skipping adjacent duplicates - no sort in this pass.
+//          lanes, dedups, writes the first 16 back to the slots and parks the
+//          rest in a pool;
+//  multi-scan: a block scan of the k per-thread counts at once gives every
+//          bucket its output offset (bucket order = (round, thread) order);
+//  pass B: stream each sorted bucket to out[offset], skipping adjacent
+//          duplicates (predicated stores, no sort).  Adjacent lanes write
+//          adjacent buckets, so a warp's stores cover a ~1 KB window.
 __device__ __forceinline__ void cswap2(uint32_t& a, uint32_t& b) {
     const uint32_t x = __vminu2(a, b), y = __vmaxu2(a, b);
     a = x;
     b = y;
 }
-__device__ __forceinline__ void sort8x2(uint32_t (&v)[8]) {  // Batcher odd-even merge sort, 19 comparators
-    cswap2(v[0], v[1]); cswap2(v[2], v[3]); cswap2(v[4], v[5]); cswap2(v[6], v[7]);
-    cswap2(v[0], v[2]); cswap2(v[1], v[3]); cswap2(v[4], v[6]); cswap2(v[5], v[7]);
-    cswap2(v[1], v[2]); cswap2(v[5], v[6]);
-    cswap2(v[0], v[4]); cswap2(v[1], v[5]); cswap2(v[2], v[6]); cswap2(v[3], v[7]);
-    cswap2(v[2], v[4]); cswap2(v[3], v[5]);
-    cswap2(v[1], v[2]); cswap2(v[3], v[4]); cswap2(v[5], v[6]);
+__device__ __forceinline__ void sort16x2(uint32_t (&v)[16]) {  // Batcher odd-even merge sort, 63 comparators
+    cswap2(v[0], v[1]); cswap2(v[2], v[3]); cswap2(v[0], v[2]); cswap2(v[1], v[3]); cswap2(v[1], v[2]);
+    cswap2(v[4], v[5]); cswap2(v[6], v[7]); cswap2(v[4], v[6]); cswap2(v[5], v[7]); cswap2(v[5], v[6]);
+    cswap2(v[0], v[4]); cswap2(v[2], v[6]); cswap2(v[2], v[4]); cswap2(v[1], v[5]); cswap2(v[3], v[7]);
+    cswap2(v[3], v[5]); cswap2(v[1], v[2]); cswap2(v[3], v[4]); cswap2(v[5], v[6]);
+    cswap2(v[8], v[9]); cswap2(v[10], v[11]); cswap2(v[8], v[10]); cswap2(v[9], v[11]); cswap2(v[9], v[10]);
+    cswap2(v[12], v[13]); cswap2(v[14], v[15]); cswap2(v[12], v[14]); cswap2(v[13], v[15]); cswap2(v[13], v[14]);
+    cswap2(v[8], v[12]); cswap2(v[10], v[14]); cswap2(v[10], v[12]); cswap2(v[9], v[13]); cswap2(v[11], v[15]);
+    cswap2(v[11], v[13]); cswap2(v[9], v[10]); cswap2(v[11], v[12]); cswap2(v[13], v[14]);
+    cswap2(v[0], v[8]); cswap2(v[4], v[12]); cswap2(v[4], v[8]); cswap2(v[2], v[10]); cswap2(v[6], v[14]);
+    cswap2(v[6], v[10]); cswap2(v[2], v[4]); cswap2(v[6], v[8]); cswap2(v[10], v[12]); cswap2(v[1], v[9]);
+    cswap2(v[5], v[13]); cswap2(v[5], v[9]); cswap2(v[3], v[11]); cswap2(v[7], v[15]); cswap2(v[7], v[11]);
+    cswap2(v[3], v[5]); cswap2(v[7], v[9]); cswap2(v[11], v[13]); cswap2(v[1], v[2]); cswap2(v[3], v[4]);
+    cswap2(v[5], v[6]); cswap2(v[7], v[8]); cswap2(v[9], v[10]); cswap2(v[11], v[12]); cswap2(v[13], v[14]);
 }
 __device__ __forceinline__ uint32_t vadd2(uint32_t a, uint32_t b) {  // per-16-bit-lane add (wrapping)
     uint32_t r;
     asm("add.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
     return r;
 }
+__device__ __forceinline__ void st_global_if(idx_t* p, idx_t v, bool pred) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+                 "r"(uint32_t(pred))
+                 : "memory");
+}
 constexpr uint32_t kOvfFlag = 0x80000000u;
+constexpr uint32_t kSlots = 16;
 
 template <int E>
 __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]);
 
-// dynamic smem: tab[MAXB] uint4 | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | ovl[OVCAP] |
-//               pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | s_cnt[THREADS]
+// dynamic smem: tabw[8*MAXB] | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | ovl[OVCAP] |
+//               pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP]
 // (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
 // which are dead once the products are inserted: BATCH * 3 >= THREADS)
 template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU>
@@ -349,24 +367,26 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
                 uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
     constexpr int NW = THREADS / 32;
+    constexpr uint32_t KMAX = (MAXB + THREADS - 1) / THREADS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    uint4* tab4 = reinterpret_cast<uint4*>(smem_raw);
+    uint32_t* tabw = reinterpret_cast<uint32_t*>(smem_raw);
     uint16_t* tab16 = reinterpret_cast<uint16_t*>(smem_raw);
-    uint32_t* bmw = reinterpret_cast<uint32_t*>(smem_raw);  // bitmap-mode view: MAXB * 5 words
-    uint32_t* bcnt = reinterpret_cast<uint32_t*>(smem_raw + MAXB * sizeof(uint4));
+    uint32_t* bmw = tabw;  // bitmap-mode view: MAXB * 9 words
+    uint32_t* bcnt = tabw + 8 * MAXB;
     const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(bcnt + MAXB);
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(sd_ptr + BATCH);
     idx_t* ovl = sd_end + BATCH;
     uint16_t* pool = reinterpret_cast<uint16_t*>(ovl + OVCAP);
-    uint32_t* obl = reinterpret_cast<uint32_t*>(pool + OVCAP);  // OVCAP even
+    uint32_t* obl = reinterpret_cast<uint32_t*>(pool + OVCAP);
     uint32_t* obcnt = obl + OBCAP;
-    uint32_t* s_cnt = obcnt + OBCAP;
     uint32_t* wbuf = reinterpret_cast<uint32_t*>(sd_ptr);
     static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0, "hash bin layout");
     __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
+    __shared__ uint32_t s_wt[KMAX][NW], s_base[KMAX + 1];
     __shared__ uint32_t s_item, s_flag, s_novf, s_nob, s_pool;
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
+    const uint32_t lt = (1u << lane) - 1u;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
     PROBE_DECL
     for (;;) {
@@ -393,10 +413,10 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         // nb buckets of width W <= 65535 (16-bit offsets); too wide a span for the
         // table goes to the bitmap bin
         const uint64_t nbw = (span + 65534) / 65535;
-        const uint32_t nb = uint32_t(min(max(max(uint64_t((u + 3) / 4), nbw), uint64_t(1)), uint64_t(MAXB)));
+        const uint32_t nb = uint32_t(min(max(max(uint64_t((u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB)));
         const uint64_t words = (span + 31) >> 5;
         idx_t* out = scratch + soff[r];
-        if (words <= 5ull * nb) {  // the span bitmap is no larger than the table
+        if (words <= 9ull * nb) {  // the span bitmap is no larger than the table
             const uint32_t nw = uint32_t(words);
             fill_words(bmw, nw, 0u, THREADS);
             __syncthreads();
@@ -416,7 +436,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         }
         const uint32_t W = uint32_t((span + nb - 1) / nb);
         const uint64_t M16 = ((((uint64_t(1) << 48) + W - 1) / W) << 16);  // ceil(2^48 / W) << 16
-        fill_words(reinterpret_cast<uint32_t*>(tab4), nb * 4, 0xFFFFFFFFu, THREADS);
+        for (uint32_t w = 0; w < 8; ++w) fill_words(tabw + w * MAXB, nb, 0xFFFFFFFFu, THREADS);
         fill_words(bcnt, nb, 0u, THREADS);
         __syncthreads();
         PROBE(2);
@@ -424,8 +444,8 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             const uint64_t d = uint64_t(c - clo);
             const uint32_t b = uint32_t(__umul64hi(d, M16));  // floor(d / W), exact for W < 2^16
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
-            if (slot < 8) {
-                tab16[b * 8 + slot] = uint16_t(uint32_t(d) - b * W);
+            if (slot < kSlots) {
+                tab16[((slot >> 1) * MAXB + b) * 2 + (slot & 1)] = uint16_t(uint32_t(d) - b * W);
             } else {
                 const uint32_t i = atomicAdd(&s_novf, 1u);
                 if (i < OVCAP) ovl[i] = c; else s_flag = 1;
@@ -437,56 +457,53 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             continue;
         }
         PROBE(4);
-        // ---- pass A: sort pairs of buckets in 16x2 SIMD, count distinct values
-        const uint32_t k = 2 * ((nb + 2 * THREADS - 1) / (2 * THREADS));
-        const uint32_t b0 = min(threadIdx.x * k, nb), b1 = min(b0 + k, nb);
-        uint32_t cnt = 0;
-        for (uint32_t b = b0; b < b1; b += 2) {
-            const bool two = b + 1 < b1;
-            const uint32_t n0 = bcnt[b], n1 = two ? bcnt[b + 1] : 0u;
-            uint4 w0 = tab4[b];
-            uint4 w1 = two ? tab4[b + 1] : make_uint4(~0u, ~0u, ~0u, ~0u);
-            if (n0 > 8 || n1 > 8) {  // rare: list the overflowing bucket(s), sort the rest
-                if (n0 > 8) {
-                    const uint32_t j = atomicAdd(&s_nob, 1u);
-                    if (j < OBCAP) obl[j] = b; else s_flag = 1;
-                    bcnt[b] = kOvfFlag | j;
-                    w0 = make_uint4(~0u, ~0u, ~0u, ~0u);
-                }
-                if (n1 > 8) {
-                    const uint32_t j = atomicAdd(&s_nob, 1u);
-                    if (j < OBCAP) obl[j] = b + 1; else s_flag = 1;
-                    bcnt[b + 1] = kOvfFlag | j;
-                    w1 = make_uint4(~0u, ~0u, ~0u, ~0u);
-                }
-            }
-            // x[i] = (slot i of bucket b+1) << 16 | (slot i of bucket b)
-            uint32_t x[8];
-            x[0] = __byte_perm(w0.x, w1.x, 0x5410); x[1] = __byte_perm(w0.x, w1.x, 0x7632);
-            x[2] = __byte_perm(w0.y, w1.y, 0x5410); x[3] = __byte_perm(w0.y, w1.y, 0x7632);
-            x[4] = __byte_perm(w0.z, w1.z, 0x5410); x[5] = __byte_perm(w0.z, w1.z, 0x7632);
-            x[6] = __byte_perm(w0.w, w1.w, 0x5410); x[7] = __byte_perm(w0.w, w1.w, 0x7632);
-            sort8x2(x);
-            // adjacent equal pairs: max(x_i, x_{i-1} + 1) - x_i is 1 iff x_i == x_{i-1}
-            // (an empty 0xFFFF predecessor wraps to 0 and counts nothing)
-            uint32_t smax = 0, sx = 0;
+        // ---- pass A: sort pairs of this thread's buckets in 16x2 SIMD ----------
+        uint32_t c[KMAX];  // distinct values per owned bucket (overflow: filled in later)
 #pragma unroll
-            for (int i = 1; i < 8; ++i) {
-                smax = vadd2(smax, __vmaxu2(x[i], vadd2(x[i - 1], 0x00010001u)));
-                sx = vadd2(sx, x[i]);
+        for (uint32_t i = 0; i < KMAX; i += 2) {
+            const uint32_t ba = threadIdx.x + i * THREADS, bb = ba + THREADS;
+            const bool va = ba < nb, vb = i + 1 < KMAX && bb < nb;
+            c[i] = 0;
+            if (i + 1 < KMAX) c[i + 1] = 0;
+            if (!va) continue;
+            uint32_t na = bcnt[ba], nbb = vb ? bcnt[bb] : 0u;
+            if (na > kSlots) {
+                const uint32_t j = atomicAdd(&s_nob, 1u);
+                if (j < OBCAP) obl[j] = ba; else s_flag = 1;
+                bcnt[ba] = kOvfFlag | j;
             }
-            const uint32_t d2 = vadd2(smax, vadd2(~sx, 0x00010001u));  // smax - sx per 16-bit lane
-            const uint32_t v0 = n0 > 8 ? 0u : n0, v1 = n1 > 8 ? 0u : n1;
-            cnt += v0 - (d2 & 0xFFFFu) + v1 - (d2 >> 16);
-            uint4 s0, s1;
-            s0.x = __byte_perm(x[0], x[1], 0x5410); s1.x = __byte_perm(x[0], x[1], 0x7632);
-            s0.y = __byte_perm(x[2], x[3], 0x5410); s1.y = __byte_perm(x[2], x[3], 0x7632);
-            s0.z = __byte_perm(x[4], x[5], 0x5410); s1.z = __byte_perm(x[4], x[5], 0x7632);
-            s0.w = __byte_perm(x[6], x[7], 0x5410); s1.w = __byte_perm(x[6], x[7], 0x7632);
-            if (n0 <= 8) tab4[b] = s0;
-            if (two && n1 <= 8) tab4[b + 1] = s1;
+            if (nbb > kSlots) {
+                const uint32_t j = atomicAdd(&s_nob, 1u);
+                if (j < OBCAP) obl[j] = bb; else s_flag = 1;
+                bcnt[bb] = kOvfFlag | j;
+            }
+            const bool sa = na <= kSlots, sb = vb && nbb <= kSlots;
+            uint32_t x[16];
+#pragma unroll
+            for (int w = 0; w < 8; ++w) {
+                const uint32_t wa = sa ? tabw[w * MAXB + ba] : ~0u;
+                const uint32_t wb = sb ? tabw[w * MAXB + bb] : ~0u;
+                x[2 * w] = __byte_perm(wa, wb, 0x5410);      // slot 2w of a | slot 2w of b
+                x[2 * w + 1] = __byte_perm(wa, wb, 0x7632);  // slot 2w+1
+            }
+            sort16x2(x);
+            // adjacent equal pairs: max(x_i, x_{i-1}+1) - x_i is 1 iff x_i == x_{i-1}
+            // (an empty 0xFFFF predecessor wraps to 0 and counts nothing); the
+            // per-half differences are >= 0, so a plain 32-bit sum keeps them apart
+            uint32_t dsum = 0;
+#pragma unroll
+            for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
+            if (sa) {
+                c[i] = na - (dsum & 0xFFFFu);
+#pragma unroll
+                for (int w = 0; w < 8; ++w) tabw[w * MAXB + ba] = __byte_perm(x[2 * w], x[2 * w + 1], 0x5410);
+            }
+            if (sb) {
+                c[i + 1] = nbb - (dsum >> 16);
+#pragma unroll
+                for (int w = 0; w < 8; ++w) tabw[w * MAXB + bb] = __byte_perm(x[2 * w], x[2 * w + 1], 0x7632);
+            }
         }
-        s_cnt[threadIdx.x] = cnt;
         __syncthreads();
         const uint32_t nob = s_nob;
         if (s_flag) {
@@ -498,18 +515,17 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             // ---- overflow buckets: one warp each, <= 32 values sorted across lanes
             const uint32_t novf = s_novf;
             uint32_t* wb = wbuf + wib * 32;
-            const uint32_t lt = (1u << lane) - 1u;
             for (uint32_t j = wib; j < nob; j += NW) {
                 const uint32_t b = obl[j];
                 const idx_t base = clo + b * W;
-                uint32_t filled = 8;
+                uint32_t filled = kSlots;
                 for (uint32_t i0 = 0; i0 < novf; i0 += 32) {
                     const uint32_t i = i0 + lane;
-                    const idx_t c = i < novf ? ovl[i] : kEmpty;
-                    const bool match = c != kEmpty && uint32_t(__umul64hi(uint64_t(c - clo), M16)) == b;
+                    const idx_t cv = i < novf ? ovl[i] : kEmpty;
+                    const bool match = cv != kEmpty && uint32_t(__umul64hi(uint64_t(cv - clo), M16)) == b;
                     const uint32_t m = __ballot_sync(FULL, match);
                     const uint32_t rank = filled + __popc(m & lt);
-                    if (match && rank < 32) wb[rank] = c;
+                    if (match && rank < 32) wb[rank] = cv;
                     filled += __popc(m);
                 }
                 __syncwarp();
@@ -518,28 +534,27 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                     continue;
                 }
                 idx_t xv[1];
-                xv[0] = lane < 8 ? base + tab16[b * 8 + lane] : (lane < filled ? wb[lane] : kEmpty);
+                xv[0] = lane < kSlots ? base + tab16[((lane >> 1) * MAXB + b) * 2 + (lane & 1)]
+                                      : (lane < filled ? wb[lane] : kEmpty);
                 __syncwarp();
                 warp_bitonic_sort<1>(xv);
                 const idx_t prev = __shfl_up_sync(FULL, xv[0], 1);
                 const bool uniq = xv[0] != kEmpty && (lane == 0 || xv[0] != prev);
                 const uint32_t um = __ballot_sync(FULL, uniq);
                 const uint32_t m = __popc(um), rank = __popc(um & lt);
-                // the first 8 distinct values go back to the bucket's slots
+                // the first 16 distinct values go back to the bucket's slots
                 // (0xFFFF-padded), the rest to the pool (extras <= list entries)
-                const uint32_t extras = m > 8 ? m - 8 : 0u;
+                const uint32_t extras = m > kSlots ? m - kSlots : 0u;
                 uint32_t off = 0;
                 if (lane == 0 && extras) off = atomicAdd(&s_pool, extras);
                 off = __shfl_sync(FULL, off, 0);
                 if (uniq) {
                     const uint16_t o = uint16_t(xv[0] - base);
-                    if (rank < 8) tab16[b * 8 + rank] = o; else pool[off + rank - 8] = o;
+                    if (rank < kSlots) tab16[((rank >> 1) * MAXB + b) * 2 + (rank & 1)] = o;
+                    else pool[off + rank - kSlots] = o;
                 }
-                if (lane < 8 && lane >= m) tab16[b * 8 + lane] = 0xFFFFu;
-                if (lane == 0) {
-                    obcnt[j] = (extras << 16) | off;
-                    atomicAdd(&s_cnt[b / k], m);
-                }
+                if (lane < kSlots && lane >= m) tab16[((lane >> 1) * MAXB + b) * 2 + (lane & 1)] = 0xFFFFu;
+                if (lane == 0) obcnt[j] = (m << 16) | off;
             }
             __syncthreads();
             if (s_flag) {
@@ -547,31 +562,64 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 __syncthreads();
                 continue;
             }
+#pragma unroll
+            for (uint32_t i = 0; i < KMAX; ++i) {
+                const uint32_t b = threadIdx.x + i * THREADS;
+                if (b < nb) {
+                    const uint32_t n = bcnt[b];
+                    if (n & kOvfFlag) c[i] = obcnt[n & ~kOvfFlag] >> 16;
+                }
+            }
         }
         PROBE(5);
-        uint64_t total;
-        uint32_t pos = uint32_t(block_exclusive_scan<uint64_t>(s_cnt[threadIdx.x], s_scan, &total));
-        PROBE(6);
-        // ---- pass B: stream the sorted buckets, skipping adjacent duplicates
-        for (uint32_t b = b0; b < b1; ++b) {
-            const uint32_t n = bcnt[b];
-            const idx_t base = clo + b * W;
-            const uint4 w = tab4[b];
-            const uint32_t q[4] = {w.x, w.y, w.z, w.w};
-            uint32_t prev = 0xFFFFu;
+        // ---- multi-scan: output offset of every owned bucket --------------------
+        uint32_t inc[KMAX];
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                const uint32_t v = (q[i >> 1] >> ((i & 1) * 16)) & 0xFFFFu;
-                if (v != 0xFFFFu && v != prev) out[pos++] = base + v;
-                prev = v;
+        for (uint32_t i = 0; i < KMAX; ++i) {
+            inc[i] = warp_inclusive_scan(c[i]);
+            if (lane == 31) s_wt[i][wib] = inc[i];
+        }
+        __syncthreads();
+        if (wib == 0) {
+            uint32_t carry = 0;
+#pragma unroll
+            for (uint32_t i = 0; i < KMAX; ++i) {
+                const uint32_t v = lane < NW ? s_wt[i][lane] : 0u;
+                const uint32_t vi = warp_inclusive_scan(v);
+                if (lane < NW) s_wt[i][lane] = carry + vi - v;
+                carry += __shfl_sync(FULL, vi, 31);
+            }
+            if (lane == 0) s_base[KMAX] = carry;
+        }
+        __syncthreads();
+        PROBE(6);
+        // ---- pass B: stream the sorted buckets, skipping adjacent duplicates ---
+#pragma unroll
+        for (uint32_t i = 0; i < KMAX; ++i) {
+            const uint32_t b = threadIdx.x + i * THREADS;
+            if (b >= nb) continue;
+            idx_t* o = out + (s_wt[i][wib] + inc[i] - c[i]);
+            const idx_t base = clo + b * W;
+            const uint32_t n = bcnt[b];
+            uint32_t pos = 0, prev = 0xFFFFu;
+#pragma unroll
+            for (int w = 0; w < 8; ++w) {
+                const uint32_t q = tabw[w * MAXB + b];
+                const uint32_t v0 = q & 0xFFFFu, v1 = q >> 16;
+                const bool k0 = v0 != 0xFFFFu && v0 != prev;
+                st_global_if(o + pos, base + v0, k0);
+                pos += k0;
+                const bool k1 = v1 != 0xFFFFu && v1 != v0;
+                st_global_if(o + pos, base + v1, k1);
+                pos += k1;
+                prev = v1;
             }
             if (n & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
                 const uint32_t e = obcnt[n & ~kOvfFlag], m = e >> 16, off = e & 0xFFFFu;
-                for (uint32_t i = 0; i < m; ++i) out[pos + i] = base + pool[off + i];
-                pos += m;
+                for (uint32_t j = kSlots; j < m; ++j) o[j] = base + pool[off + j - kSlots];
             }
         }
-        if (threadIdx.x == 0) counts[r] = uint32_t(total);
+        if (threadIdx.x == 0) counts[r] = s_base[KMAX];
         __syncthreads();
         PROBE(7);
         PROBE_PRINT("hash", u, num_segs(src, r));
@@ -991,24 +1039,24 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
 constexpr uint32_t kDBatch = 2048;
 constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, uint32_t ovcap, uint32_t obcap) {
-    return buckets * (sizeof(uint4) + sizeof(uint32_t)) + batch * kSegBytes + ovcap * (sizeof(idx_t) + sizeof(uint16_t)) +
-           obcap * 2 * sizeof(uint32_t) + threads * sizeof(uint32_t);
+    return buckets * (8 * sizeof(uint32_t) + sizeof(uint32_t)) + batch * kSegBytes +
+           ovcap * (sizeof(idx_t) + sizeof(uint16_t)) + obcap * 2 * sizeof(uint32_t);
 }
 #define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U)                                           \
     constexpr int NAME##_T = T, NAME##_PERSM = PERSM, NAME##_U = U;                                \
-    constexpr uint32_t NAME##_B = uint32_t(UB / 4), NAME##_OVCAP = OVCAP, NAME##_OBCAP = OBCAP,     \
+    constexpr uint32_t NAME##_B = uint32_t(UB / 8), NAME##_OVCAP = OVCAP, NAME##_OBCAP = OBCAP,     \
                        NAME##_BATCH = BATCH;                                                       \
-    constexpr size_t NAME##_SMEM = hash_smem(T, BATCH, uint32_t(UB / 4), OVCAP, OBCAP);            \
-    static_assert(PERSM * (NAME##_SMEM + 1024 + 600) <= 228 * 1024, #NAME " residency");          \
+    constexpr size_t NAME##_SMEM = hash_smem(T, BATCH, uint32_t(UB / 8), OVCAP, OBCAP);            \
+    static_assert(PERSM * (NAME##_SMEM + 1024 + 1200) <= 228 * 1024, #NAME " residency");         \
     static_assert(PERSM * T <= 2048, #NAME " threads");
 // <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread>
-// (expected per row at mean load 4: list ~ub/130, buckets ~ub/190)
-HBIN(H1, 128, kH1, 64, 16, 256, 12, 4)
-HBIN(H2, 128, kH2, 64, 32, 256, 12, 4)
-HBIN(H3, 256, kH3, 128, 64, 384, 6, 4)
-HBIN(H4, 256, kH4, 256, 128, 256, 4, 8)
-HBIN(H5, 512, kH5, 384, 256, 256, 2, 8)
-HBIN(H6, 1024, kH6, 768, 512, 384, 1, 8)
+// (expected per row at mean load 8 with 16 slots: list ~ub/1500, buckets ~ub/2000)
+HBIN(H1, 128, kH1, 32, 16, 256, 10, 4)
+HBIN(H2, 128, kH2, 32, 16, 256, 10, 4)
+HBIN(H3, 256, kH3, 64, 32, 384, 5, 4)
+HBIN(H4, 256, kH4, 64, 32, 256, 4, 8)
+HBIN(H5, 512, kH5, 128, 64, 256, 2, 8)
+HBIN(H6, 1024, kH6, 192, 96, 384, 1, 8)
 #define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U>
 #define HASH1 HASHK(H1)
 #define HASH2 HASHK(H2)
