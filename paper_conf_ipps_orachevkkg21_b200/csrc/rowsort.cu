@@ -168,6 +168,7 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
     const uint32_t per = (n + THREADS - 1) / THREADS;
     const uint32_t b = threadIdx.x * per, e = min(b + per, n);
     uint64_t acc = 0;  // (non-empty count << 32) | product count
+#pragma unroll 1
     for (uint32_t i = b; i < e; ++i) {
         uint32_t len;
         get_seg(s, r, s0 + i, len);
@@ -176,6 +177,7 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
     uint64_t tot;
     const uint64_t ex = block_exclusive_scan<uint64_t>(acc, s_scan, &tot);
     uint32_t k = uint32_t(ex >> 32), run = uint32_t(ex);
+#pragma unroll 1
     for (uint32_t i = b; i < e; ++i) {
         uint32_t len;
         const idx_t* p = get_seg(s, r, s0 + i, len);
@@ -217,22 +219,32 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, cons
             uint32_t k = lo, end = sd_end[lo];
             const idx_t* p = sd_ptr[lo];
             idx_t v[U];
+            // consecutive products cross at most one boundary (segments are
+            // non-empty), so each step is a single predicated advance
+            if (q0 + U <= total) {
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                const uint32_t q = q0 + u;
-                v[u] = kEmpty;
-                if (q < total) {
-                    while (q >= end) {  // staged segments are non-empty
+                for (int u = 0; u < U; ++u) {
+                    const uint32_t q = q0 + u;
+                    if (u > 0 && q >= end) {
                         ++k;
                         end = sd_end[k];
                         p = sd_ptr[k];
                     }
                     v[u] = __ldg(p + q);
                 }
-            }
 #pragma unroll
-            for (int u = 0; u < U; ++u)
-                if (v[u] != kEmpty) f(v[u]);
+                for (int u = 0; u < U; ++u) f(v[u]);
+            } else {  // ragged tail of the row: rolled (keeps the kernel small)
+#pragma unroll 1
+                for (uint32_t q = q0; q < total; ++q) {
+                    if (q > q0 && q >= end) {
+                        ++k;
+                        end = sd_end[k];
+                        p = sd_ptr[k];
+                    }
+                    f(__ldg(p + q));
+                }
+            }
         }
         __syncthreads();  // descriptors are reused by the next batch
     }
@@ -289,7 +301,9 @@ __device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, 
     // p is 16-byte aligned; vector stores for the bulk
     uint4* p4 = reinterpret_cast<uint4*>(p);
     const uint4 v4 = make_uint4(v, v, v, v);
+#pragma unroll 1
     for (uint32_t i = threadIdx.x; i < n / 4; i += threads) p4[i] = v4;
+#pragma unroll 1
     for (uint32_t i = (n & ~3u) + threadIdx.x; i < n; i += threads) p[i] = v;
 }
 
@@ -301,25 +315,26 @@ __device__ __forceinline__ void fill_words(uint32_t* p, uint32_t n, uint32_t v, 
 // store - no probing, no CAS, no lane divergence; duplicates are dropped at
 // emission.  nb = ub/8 buckets (mean load <= 8, 4.5 bytes of smem per
 // product); a product arriving at a full bucket (p ~ 0.4%) is appended to a
-// small overflow list.  The table is stored word-transposed: word w (slots
-// 2w, 2w+1) of bucket b at tabw[w*MAXB + b], so a warp reading 32 adjacent
-// buckets touches 32 banks.
+// small overflow list.  The table is slot-major: slot s of bucket b at
+// tab16[s*MAXB + b], so one 32-bit word holds slot s of the bucket pair
+// (2m, 2m+1) - exactly one 16x2 SIMD register of the pair's sort.
 //
-// Emission: thread t owns buckets t, t+T, t+2T, ... (k <= KMAX of them).
-//  pass A: two buckets at a time in 16x2 SIMD registers (VIMNMX.U16x2): a
-//          16-input Batcher network (63 comparators) sorts both, the sorted
-//          slots are written back, the distinct values are counted (n_valid
-//          minus adjacent equal pairs, via max(x_i, x_{i-1}+1) - x_i summed
-//          in 32-bit arithmetic).  A bucket that overflowed is listed instead;
+// Emission: thread t owns bucket pairs t, t+T, t+2T, ... (KP of them).
+//  pass A: per pair, 16 conflict-free LDS.32 give x[s] = (slot s of 2m+1,
+//          slot s of 2m); a 16-input Batcher network (63 comparators) on
+//          VIMNMX.U16x2 sorts both buckets, the sorted slots are written
+//          back, the distinct values are counted (n_valid minus adjacent
+//          equal pairs, via max(x_i, x_{i-1}+1) - x_i summed in 32-bit
+//          arithmetic).  A bucket that overflowed is listed instead;
 //  overflow: one warp per listed bucket gathers its 16 slots and its list
 //          entries (ballot over the list), bitonic-sorts <= 32 values across
 //          lanes, dedups, writes the first 16 back to the slots and parks the
 //          rest in a pool;
-//  multi-scan: a block scan of the k per-thread counts at once gives every
-//          bucket its output offset (bucket order = (round, thread) order);
-//  pass B: stream each sorted bucket to out[offset], skipping adjacent
+//  multi-scan: a block scan of the KP per-thread pair counts at once gives
+//          every pair its output offset (pair order = (round, thread) order);
+//  pass B: stream each sorted pair to out[offset], skipping adjacent
 //          duplicates (predicated stores, no sort).  Adjacent lanes write
-//          adjacent buckets, so a warp's stores cover a ~1 KB window.
+//          adjacent pairs, so a warp's stores cover a ~2 KB window.
 __device__ __forceinline__ void cswap2(uint32_t& a, uint32_t& b) {
     const uint32_t x = __vminu2(a, b), y = __vmaxu2(a, b);
     a = x;
@@ -345,10 +360,19 @@ __device__ __forceinline__ uint32_t vadd2(uint32_t a, uint32_t b) {  // per-16-b
     asm("add.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
     return r;
 }
-__device__ __forceinline__ void st_global_if(idx_t* p, idx_t v, bool pred) {
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
-                 "r"(uint32_t(pred))
-                 : "memory");
+// o[pos] = base + v and pos += 1 if v is a valid slot (!= 0xFFFF) distinct from prev
+__device__ __forceinline__ void emit_if(idx_t* o, uint32_t& pos, uint32_t base, uint32_t v, uint32_t prev) {
+    asm volatile(
+        "{\n\t.reg .pred q;\n\t.reg .u64 a;\n\t.reg .u32 x;\n\t"
+        "setp.ne.u32 q, %2, %3;\n\t"
+        "setp.ne.and.u32 q, %2, 65535, q;\n\t"
+        "mad.wide.u32 a, %0, 4, %4;\n\t"
+        "add.u32 x, %1, %2;\n\t"
+        "@q st.global.u32 [a], x;\n\t"
+        "@q add.u32 %0, %0, 1;\n\t}"
+        : "+r"(pos)
+        : "r"(base), "r"(v), "r"(prev), "l"(o)
+        : "memory");
 }
 constexpr uint32_t kOvfFlag = 0x80000000u;
 constexpr uint32_t kSlots = 16;
@@ -356,8 +380,8 @@ constexpr uint32_t kSlots = 16;
 template <int E>
 __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]);
 
-// dynamic smem: tabw[8*MAXB] | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | ovl[OVCAP] |
-//               pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP]
+// dynamic smem: tab16[16*MAXB] | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | ovl[OVCAP] |
+//               pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | poff[MAXB/2]
 // (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
 // which are dead once the products are inserted: BATCH * 3 >= THREADS)
 template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU>
@@ -367,9 +391,10 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
                 uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
     constexpr int NW = THREADS / 32;
-    constexpr uint32_t KMAX = (MAXB + THREADS - 1) / THREADS;
+    constexpr uint32_t MP = MAXB / 2;                      // bucket pairs
+    constexpr uint32_t KP = (MP + THREADS - 1) / THREADS;  // pairs per thread
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    uint32_t* tabw = reinterpret_cast<uint32_t*>(smem_raw);
+    uint32_t* tabw = reinterpret_cast<uint32_t*>(smem_raw);  // word s*MP + m = slot s of pair m
     uint16_t* tab16 = reinterpret_cast<uint16_t*>(smem_raw);
     uint32_t* bmw = tabw;  // bitmap-mode view: MAXB * 9 words
     uint32_t* bcnt = tabw + 8 * MAXB;
@@ -379,11 +404,12 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     uint16_t* pool = reinterpret_cast<uint16_t*>(ovl + OVCAP);
     uint32_t* obl = reinterpret_cast<uint32_t*>(pool + OVCAP);
     uint32_t* obcnt = obl + OBCAP;
+    uint32_t* poff = obcnt + OBCAP;  // [MP] output offset of each bucket pair
     uint32_t* wbuf = reinterpret_cast<uint32_t*>(sd_ptr);
     static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0, "hash bin layout");
     __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_wt[KMAX][NW], s_base[KMAX + 1];
+    __shared__ uint32_t s_wt[KP][NW], s_total;
     __shared__ uint32_t s_item, s_flag, s_novf, s_nob, s_pool;
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
@@ -411,9 +437,10 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         }
         const uint64_t span = uint64_t(chi) - clo + 1;
         // nb buckets of width W <= 65535 (16-bit offsets); too wide a span for the
-        // table goes to the bitmap bin
+        // table goes to the bitmap bin.  nb is even (buckets are sorted in pairs).
         const uint64_t nbw = (span + 65534) / 65535;
-        const uint32_t nb = uint32_t(min(max(max(uint64_t((u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB)));
+        const uint32_t nb =
+            (uint32_t(min(max(max(uint64_t((u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB))) + 1) & ~1u;
         const uint64_t words = (span + 31) >> 5;
         idx_t* out = scratch + soff[r];
         if (words <= 9ull * nb) {  // the span bitmap is no larger than the table
@@ -434,18 +461,26 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             __syncthreads();
             continue;
         }
+        // bucket width W (> 288 here: smaller spans took the bitmap) and an exact
+        // 32-bit reciprocal: d < nb*W < 2^29, M = ceil(2^(32+l) / W) with
+        // 2^(l+3) >= W gives floor(d / W) = umulhi(d, M) >> l (M < 2^30)
         const uint32_t W = uint32_t((span + nb - 1) / nb);
-        const uint64_t M16 = ((((uint64_t(1) << 48) + W - 1) / W) << 16);  // ceil(2^48 / W) << 16
-        for (uint32_t w = 0; w < 8; ++w) fill_words(tabw + w * MAXB, nb, 0xFFFFFFFFu, THREADS);
+        const uint32_t l = (32 - __clz(W - 1)) - 3;
+        const uint32_t M = uint32_t(((uint64_t(1) << (32 + l)) + W - 1) / W);
+        const uint32_t np = nb / 2;
+#pragma unroll 1
+        for (uint32_t sl = 0; sl < kSlots; ++sl)
+#pragma unroll 1
+            for (uint32_t i = threadIdx.x; i < np; i += THREADS) tabw[sl * MP + i] = 0xFFFFFFFFu;
         fill_words(bcnt, nb, 0u, THREADS);
         __syncthreads();
         PROBE(2);
         block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
-            const uint64_t d = uint64_t(c - clo);
-            const uint32_t b = uint32_t(__umul64hi(d, M16));  // floor(d / W), exact for W < 2^16
+            const uint32_t d = c - clo;
+            const uint32_t b = __umulhi(d, M) >> l;
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
             if (slot < kSlots) {
-                tab16[((slot >> 1) * MAXB + b) * 2 + (slot & 1)] = uint16_t(uint32_t(d) - b * W);
+                tab16[slot * MAXB + b] = uint16_t(d - b * W);
             } else {
                 const uint32_t i = atomicAdd(&s_novf, 1u);
                 if (i < OVCAP) ovl[i] = c; else s_flag = 1;
@@ -457,35 +492,29 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             continue;
         }
         PROBE(4);
-        // ---- pass A: sort pairs of this thread's buckets in 16x2 SIMD ----------
-        uint32_t c[KMAX];  // distinct values per owned bucket (overflow: filled in later)
-#pragma unroll
-        for (uint32_t i = 0; i < KMAX; i += 2) {
-            const uint32_t ba = threadIdx.x + i * THREADS, bb = ba + THREADS;
-            const bool va = ba < nb, vb = i + 1 < KMAX && bb < nb;
-            c[i] = 0;
-            if (i + 1 < KMAX) c[i + 1] = 0;
-            if (!va) continue;
-            uint32_t na = bcnt[ba], nbb = vb ? bcnt[bb] : 0u;
-            if (na > kSlots) {
+        // ---- pass A: sort each owned bucket pair in 16x2 SIMD ----------------
+        // (rolled loops from here on: the kernel must stay small for the I-cache)
+        // bcnt[b] becomes the bucket's distinct count, or kOvfFlag | list index
+#pragma unroll 1
+        for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
+            const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+            uint32_t keep = 0xFFFFFFFFu;  // lanes of an overflowed bucket are masked out of the sort
+            uint2 res;
+            if (nn.x > kSlots) {
                 const uint32_t j = atomicAdd(&s_nob, 1u);
-                if (j < OBCAP) obl[j] = ba; else s_flag = 1;
-                bcnt[ba] = kOvfFlag | j;
+                if (j < OBCAP) obl[j] = 2 * m; else s_flag = 1;
+                res.x = kOvfFlag | j;
+                keep &= 0xFFFF0000u;
             }
-            if (nbb > kSlots) {
+            if (nn.y > kSlots) {
                 const uint32_t j = atomicAdd(&s_nob, 1u);
-                if (j < OBCAP) obl[j] = bb; else s_flag = 1;
-                bcnt[bb] = kOvfFlag | j;
+                if (j < OBCAP) obl[j] = 2 * m + 1; else s_flag = 1;
+                res.y = kOvfFlag | j;
+                keep &= 0x0000FFFFu;
             }
-            const bool sa = na <= kSlots, sb = vb && nbb <= kSlots;
             uint32_t x[16];
 #pragma unroll
-            for (int w = 0; w < 8; ++w) {
-                const uint32_t wa = sa ? tabw[w * MAXB + ba] : ~0u;
-                const uint32_t wb = sb ? tabw[w * MAXB + bb] : ~0u;
-                x[2 * w] = __byte_perm(wa, wb, 0x5410);      // slot 2w of a | slot 2w of b
-                x[2 * w + 1] = __byte_perm(wa, wb, 0x7632);  // slot 2w+1
-            }
+            for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m] | ~keep;
             sort16x2(x);
             // adjacent equal pairs: max(x_i, x_{i-1}+1) - x_i is 1 iff x_i == x_{i-1}
             // (an empty 0xFFFF predecessor wraps to 0 and counts nothing); the
@@ -493,16 +522,12 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             uint32_t dsum = 0;
 #pragma unroll
             for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
-            if (sa) {
-                c[i] = na - (dsum & 0xFFFFu);
+            if (nn.x <= kSlots) res.x = nn.x - (dsum & 0xFFFFu);
+            if (nn.y <= kSlots) res.y = nn.y - (dsum >> 16);
+            reinterpret_cast<uint2*>(bcnt)[m] = res;
+            // an overflowed bucket keeps its raw slots for the overflow pass
 #pragma unroll
-                for (int w = 0; w < 8; ++w) tabw[w * MAXB + ba] = __byte_perm(x[2 * w], x[2 * w + 1], 0x5410);
-            }
-            if (sb) {
-                c[i + 1] = nbb - (dsum >> 16);
-#pragma unroll
-                for (int w = 0; w < 8; ++w) tabw[w * MAXB + bb] = __byte_perm(x[2 * w], x[2 * w + 1], 0x7632);
-            }
+            for (int sl = 0; sl < 16; ++sl) tabw[sl * MP + m] = (x[sl] & keep) | (tabw[sl * MP + m] & ~keep);
         }
         __syncthreads();
         const uint32_t nob = s_nob;
@@ -522,11 +547,11 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 for (uint32_t i0 = 0; i0 < novf; i0 += 32) {
                     const uint32_t i = i0 + lane;
                     const idx_t cv = i < novf ? ovl[i] : kEmpty;
-                    const bool match = cv != kEmpty && uint32_t(__umul64hi(uint64_t(cv - clo), M16)) == b;
-                    const uint32_t m = __ballot_sync(FULL, match);
-                    const uint32_t rank = filled + __popc(m & lt);
+                    const bool match = cv != kEmpty && (__umulhi(cv - clo, M) >> l) == b;
+                    const uint32_t mm = __ballot_sync(FULL, match);
+                    const uint32_t rank = filled + __popc(mm & lt);
                     if (match && rank < 32) wb[rank] = cv;
-                    filled += __popc(m);
+                    filled += __popc(mm);
                 }
                 __syncwarp();
                 if (filled > 32) {  // warp-uniform
@@ -534,27 +559,25 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                     continue;
                 }
                 idx_t xv[1];
-                xv[0] = lane < kSlots ? base + tab16[((lane >> 1) * MAXB + b) * 2 + (lane & 1)]
-                                      : (lane < filled ? wb[lane] : kEmpty);
+                xv[0] = lane < kSlots ? base + tab16[lane * MAXB + b] : (lane < filled ? wb[lane] : kEmpty);
                 __syncwarp();
                 warp_bitonic_sort<1>(xv);
                 const idx_t prev = __shfl_up_sync(FULL, xv[0], 1);
                 const bool uniq = xv[0] != kEmpty && (lane == 0 || xv[0] != prev);
                 const uint32_t um = __ballot_sync(FULL, uniq);
-                const uint32_t m = __popc(um), rank = __popc(um & lt);
+                const uint32_t mcnt = __popc(um), rank = __popc(um & lt);
                 // the first 16 distinct values go back to the bucket's slots
                 // (0xFFFF-padded), the rest to the pool (extras <= list entries)
-                const uint32_t extras = m > kSlots ? m - kSlots : 0u;
+                const uint32_t extras = mcnt > kSlots ? mcnt - kSlots : 0u;
                 uint32_t off = 0;
                 if (lane == 0 && extras) off = atomicAdd(&s_pool, extras);
                 off = __shfl_sync(FULL, off, 0);
                 if (uniq) {
                     const uint16_t o = uint16_t(xv[0] - base);
-                    if (rank < kSlots) tab16[((rank >> 1) * MAXB + b) * 2 + (rank & 1)] = o;
-                    else pool[off + rank - kSlots] = o;
+                    if (rank < kSlots) tab16[rank * MAXB + b] = o; else pool[off + rank - kSlots] = o;
                 }
-                if (lane < kSlots && lane >= m) tab16[((lane >> 1) * MAXB + b) * 2 + (lane & 1)] = 0xFFFFu;
-                if (lane == 0) obcnt[j] = (m << 16) | off;
+                if (lane < kSlots && lane >= mcnt) tab16[lane * MAXB + b] = 0xFFFFu;
+                if (lane == 0) obcnt[j] = (mcnt << 16) | off;
             }
             __syncthreads();
             if (s_flag) {
@@ -562,64 +585,75 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 __syncthreads();
                 continue;
             }
-#pragma unroll
-            for (uint32_t i = 0; i < KMAX; ++i) {
-                const uint32_t b = threadIdx.x + i * THREADS;
-                if (b < nb) {
-                    const uint32_t n = bcnt[b];
-                    if (n & kOvfFlag) c[i] = obcnt[n & ~kOvfFlag] >> 16;
-                }
-            }
         }
         PROBE(5);
-        // ---- multi-scan: output offset of every owned bucket --------------------
-        uint32_t inc[KMAX];
+        // ---- multi-scan: output offset of every owned pair -> poff[m] ----------
+        auto bucket_count = [&](uint32_t x) { return (x & kOvfFlag) ? obcnt[x & ~kOvfFlag] >> 16 : x; };
+        uint32_t cpair[KP], inc[KP];
 #pragma unroll
-        for (uint32_t i = 0; i < KMAX; ++i) {
-            inc[i] = warp_inclusive_scan(c[i]);
+        for (uint32_t i = 0; i < KP; ++i) {
+            const uint32_t m = threadIdx.x + i * THREADS;
+            cpair[i] = 0;
+            if (m < np) {
+                const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+                cpair[i] = bucket_count(nn.x) + bucket_count(nn.y);
+            }
+            inc[i] = warp_inclusive_scan(cpair[i]);
             if (lane == 31) s_wt[i][wib] = inc[i];
         }
         __syncthreads();
         if (wib == 0) {
             uint32_t carry = 0;
 #pragma unroll
-            for (uint32_t i = 0; i < KMAX; ++i) {
+            for (uint32_t i = 0; i < KP; ++i) {
                 const uint32_t v = lane < NW ? s_wt[i][lane] : 0u;
                 const uint32_t vi = warp_inclusive_scan(v);
                 if (lane < NW) s_wt[i][lane] = carry + vi - v;
                 carry += __shfl_sync(FULL, vi, 31);
             }
-            if (lane == 0) s_base[KMAX] = carry;
+            if (lane == 0) s_total = carry;
         }
         __syncthreads();
-        PROBE(6);
-        // ---- pass B: stream the sorted buckets, skipping adjacent duplicates ---
 #pragma unroll
-        for (uint32_t i = 0; i < KMAX; ++i) {
-            const uint32_t b = threadIdx.x + i * THREADS;
-            if (b >= nb) continue;
-            idx_t* o = out + (s_wt[i][wib] + inc[i] - c[i]);
-            const idx_t base = clo + b * W;
-            const uint32_t n = bcnt[b];
+        for (uint32_t i = 0; i < KP; ++i) {
+            const uint32_t m = threadIdx.x + i * THREADS;
+            if (m < np) poff[m] = s_wt[i][wib] + inc[i] - cpair[i];
+        }
+        PROBE(6);
+        // ---- pass B: stream the sorted pairs, skipping adjacent duplicates -----
+        // (each thread reads back only its own poff entries: no barrier needed)
+#pragma unroll 1
+        for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
+            idx_t* o = out + poff[m];
+            const idx_t base0 = clo + 2 * m * W, base1 = base0 + W;
+            const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+            uint32_t x[16];
+#pragma unroll
+            for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m];
             uint32_t pos = 0, prev = 0xFFFFu;
 #pragma unroll
-            for (int w = 0; w < 8; ++w) {
-                const uint32_t q = tabw[w * MAXB + b];
-                const uint32_t v0 = q & 0xFFFFu, v1 = q >> 16;
-                const bool k0 = v0 != 0xFFFFu && v0 != prev;
-                st_global_if(o + pos, base + v0, k0);
-                pos += k0;
-                const bool k1 = v1 != 0xFFFFu && v1 != v0;
-                st_global_if(o + pos, base + v1, k1);
-                pos += k1;
-                prev = v1;
+            for (int sl = 0; sl < 16; ++sl) {
+                const uint32_t v = x[sl] & 0xFFFFu;
+                emit_if(o, pos, base0, v, prev);
+                prev = v;
             }
-            if (n & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
-                const uint32_t e = obcnt[n & ~kOvfFlag], m = e >> 16, off = e & 0xFFFFu;
-                for (uint32_t j = kSlots; j < m; ++j) o[j] = base + pool[off + j - kSlots];
+            if (nn.x & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
+                const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base0 + pool[off + j - kSlots];
+            }
+            prev = 0xFFFFu;
+#pragma unroll
+            for (int sl = 0; sl < 16; ++sl) {
+                const uint32_t v = x[sl] >> 16;
+                emit_if(o, pos, base1, v, prev);
+                prev = v;
+            }
+            if (nn.y & kOvfFlag) {
+                const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base1 + pool[off + j - kSlots];
             }
         }
-        if (threadIdx.x == 0) counts[r] = s_base[KMAX];
+        if (threadIdx.x == 0) counts[r] = s_total;
         __syncthreads();
         PROBE(7);
         PROBE_PRINT("hash", u, num_segs(src, r));
@@ -1039,7 +1073,7 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
 constexpr uint32_t kDBatch = 2048;
 constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, uint32_t ovcap, uint32_t obcap) {
-    return buckets * (8 * sizeof(uint32_t) + sizeof(uint32_t)) + batch * kSegBytes +
+    return buckets * (8 * sizeof(uint32_t) + sizeof(uint32_t) + sizeof(uint16_t)) + batch * kSegBytes +
            ovcap * (sizeof(idx_t) + sizeof(uint16_t)) + obcap * 2 * sizeof(uint32_t);
 }
 #define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U)                                           \
