@@ -129,18 +129,18 @@ void exclusive_scan_u64(const uint64_t* in, uint64_t* out, size_t n);
 // union of a per-row list of column "segments" (MxM: B rows; Build /
 // Transpose: one bucket), then compact into CSR.  See DESIGN.md §4.2.
 struct SegSource {
-    // MxM mode (kind = 0): segments of row r are C[r] (if crp) then B[k] for
-    // k in A[r].  List mode (kind = 1): one segment lst[lrp[r] .. lrp[r+1]).
+    // Descriptor mode (kind = 0, MxM): row r's NON-EMPTY segments are
+    // desc[dbase[r] + r + j], j < nseg[r], each {ptr lo, ptr hi, len, end}
+    // with end = inclusive prefix of the row's segment lengths (written by
+    // the upper-bound pass: C[r] first when accumulating, then B[k] for k in
+    // A[r]).  Staging a row is then a plain copy.  List mode (kind = 1,
+    // Build / Transpose): one segment lst[lrp[r] .. lrp[r+1]).
     int kind;
-    int sorted;  // segments sorted ascending (MxM: yes; Build/Transpose buckets: no)
-    const off_t64* __restrict__ arp; const idx_t* __restrict__ aci;
-    const off_t64* __restrict__ brp; const idx_t* __restrict__ bci;
-    const off_t64* __restrict__ crp; const idx_t* __restrict__ cci;
-    const off_t64* __restrict__ lrp; const idx_t* __restrict__ lst;
-    // MxM: per A entry p the B segment as {ptr lo, ptr hi, len, 0} (written by
-    // the upper-bound pass, so staging a row costs one coalesced load per
-    // segment instead of the dependent aci -> brp chain); may be null
+    const off_t64* __restrict__ dbase;
+    const uint32_t* __restrict__ nseg;
     const uint4* __restrict__ desc;
+    const off_t64* __restrict__ lrp;
+    const idx_t* __restrict__ lst;
 };
 // ub: per-row upper bound of entries (device, nrows).  Installs the result
 // in `out` (nrows x ncols).  dedup=false promises rows are duplicate-free.

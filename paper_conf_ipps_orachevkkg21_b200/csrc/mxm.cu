@@ -20,30 +20,63 @@ constexpr int kGroup = 8;
 __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
                               const off_t64* __restrict__ crp, const idx_t* __restrict__ cci,
                               uint64_t* __restrict__ ub, uint2* __restrict__ range,
-                              uint4* __restrict__ desc) {
-    const unsigned g = threadIdx.x & (kGroup - 1);
+                              uint4* __restrict__ desc, uint32_t* __restrict__ nseg) {
+    const unsigned lane = threadIdx.x & 31, g = lane & (kGroup - 1);
+    const unsigned gshift = lane & ~(kGroup - 1);  // first lane of this row's group
     const size_t ngroups = (size_t(gridDim.x) * blockDim.x) / kGroup;
     // warp-uniform loop: every lane of a warp runs the same trip count
     for (size_t rb = (blockIdx.x * size_t(blockDim.x) + (threadIdx.x & ~31u)) / kGroup; rb < A.nrows;
          rb += ngroups) {
-        const size_t r = rb + (threadIdx.x & 31) / kGroup;
+        const size_t r = rb + lane / kGroup;
         const bool valid = r < A.nrows;
         uint64_t s = 0;
         off_t64 b = 0, e = 0;
+        uint32_t cn = 0, cl = 0;  // running non-empty count / product prefix of the row
+        uint4* drow = nullptr;
         if (valid) {
             b = A.rowptr[r];
             e = A.rowptr[r + 1];
-            for (off_t64 p = b + g; p < e; p += kGroup) {
-                idx_t k = A.colidx[p];
-                const off_t64 x = brp[k], y = brp[k + 1];
-                s += y - x;
-                const uint64_t ptr = reinterpret_cast<uint64_t>(bci + x);
-                desc[p] = make_uint4(uint32_t(ptr), uint32_t(ptr >> 32), uint32_t(y - x), 0u);
+            drow = desc + (b + r);  // room for the C[r] segment in front
+            if (crp) {
+                const off_t64 cb = crp[r];
+                const uint32_t lc = uint32_t(crp[r + 1] - cb);
+                if (lc) {
+                    if (g == 0) {
+                        const uint64_t ptr = reinterpret_cast<uint64_t>(cci + cb);
+                        drow[0] = make_uint4(uint32_t(ptr), uint32_t(ptr >> 32), lc, lc);
+                    }
+                    cn = 1;
+                    cl = lc;
+                    s = g == 0 ? lc : 0;
+                }
             }
+        }
+        const uint32_t trips = __reduce_max_sync(0xffffffffu, valid ? uint32_t((e - b + kGroup - 1) / kGroup) : 0u);
+        for (uint32_t it = 0; it < trips; ++it) {
+            const off_t64 p = b + it * kGroup + g;
+            uint32_t len = 0;
+            uint64_t ptr = 0;
+            if (valid && p < e) {
+                const idx_t k = A.colidx[p];
+                const off_t64 x = brp[k], y = brp[k + 1];
+                len = uint32_t(y - x);
+                ptr = reinterpret_cast<uint64_t>(bci + x);
+            }
+            s += len;
+            // compacted position and inclusive length prefix inside the group
+            const uint32_t m = (__ballot_sync(0xffffffffu, len > 0) >> gshift) & 0xFFu;
+            uint32_t inc = len;
+#pragma unroll
+            for (int d = 1; d < kGroup; d <<= 1) {
+                const uint32_t t = __shfl_up_sync(0xffffffffu, inc, d, kGroup);
+                if (g >= unsigned(d)) inc += t;
+            }
+            if (len) drow[cn + __popc(m & ((1u << g) - 1u))] = make_uint4(uint32_t(ptr), uint32_t(ptr >> 32), len, cl + inc);
+            cn += __popc(m);
+            cl += __shfl_sync(0xffffffffu, inc, kGroup - 1, kGroup);
         }
 #pragma unroll
         for (int d = kGroup / 2; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d, kGroup);
-        if (valid && crp) s += crp[r + 1] - crp[r];
         // column span of the row (segments are sorted: first / last entries),
         // used by the hash and bitmap bins of the row engine
         const bool need = valid && s > kRangeMinUb;
@@ -69,6 +102,7 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
         }
         if (valid && g == 0) {
             ub[r] = s;
+            nseg[r] = cn;
             if (need) range[r] = make_uint2(lo, hi);
         }
     }
@@ -91,25 +125,21 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     trace_mark("mxm start");
     DevBuf<uint64_t> ub(m);
     DevBuf<uint2> range(m);
-    DevBuf<uint4> desc(A->nnz);
+    DevBuf<uint4> desc(A->nnz + m);  // per row: C[r] (accumulate) + non-empty B rows
+    DevBuf<uint32_t> nseg(m);
     const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
                                                        uint64_t(ctx().num_sms) * 16);
     const off_t64* crp = accumulate ? C->rowptr : nullptr;
     int tk = ktime_begin("mxm_ub", ctx().stream);
     mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, crp,
-                                                  accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p);
+                                                  accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p, nseg.p);
     ktime_end(tk);
     count_launch();
     check_launch("mxm_ub_kernel");
     SegSource src{};
     src.kind = 0;
-    src.sorted = 1;
-    src.arp = A->rowptr;
-    src.aci = A->colidx;
-    src.brp = B->rowptr;
-    src.bci = B->colidx;
-    src.crp = crp;
-    src.cci = accumulate ? C->colidx : nullptr;
+    src.dbase = A->rowptr;
+    src.nseg = nseg.p;
     src.desc = desc.p;
     // the engine writes fresh storage and only then installs it into C, so
     // C may alias A and/or B

@@ -94,7 +94,7 @@ __device__ __forceinline__ int bin_of(uint64_t ub) {
 // ---- segment access --------------------------------------------------------
 __device__ __forceinline__ uint32_t num_segs(const SegSource& s, idx_t r) {
     if (s.kind == 1) return 1;
-    return uint32_t(s.arp[r + 1] - s.arp[r]) + (s.crp ? 1u : 0u);
+    return s.nseg[r];
 }
 
 __device__ __forceinline__ const idx_t* get_seg(const SegSource& s, idx_t r, uint32_t j, uint32_t& len) {
@@ -103,23 +103,9 @@ __device__ __forceinline__ const idx_t* get_seg(const SegSource& s, idx_t r, uin
         len = uint32_t(s.lrp[r + 1] - b);
         return s.lst + b;
     }
-    if (s.crp) {
-        if (j == 0) {
-            off_t64 b = s.crp[r];
-            len = uint32_t(s.crp[r + 1] - b);
-            return s.cci + b;
-        }
-        --j;
-    }
-    if (s.desc) {
-        const uint4 d = s.desc[s.arp[r] + j];
-        len = d.z;
-        return reinterpret_cast<const idx_t*>((uint64_t(d.y) << 32) | d.x);
-    }
-    idx_t k = s.aci[s.arp[r] + j];
-    off_t64 b = s.brp[k];
-    len = uint32_t(s.brp[k + 1] - b);
-    return s.bci + b;
+    const uint4 d = s.desc[s.dbase[r] + r + j];
+    len = d.z;
+    return reinterpret_cast<const idx_t*>((uint64_t(d.y) << 32) | d.x);
 }
 
 // Flattened warp gather: every lane holds one segment (p, len); the warp
@@ -157,40 +143,35 @@ __device__ __forceinline__ uint32_t warp_flat(const idx_t* p, uint32_t len, F&& 
 }
 
 // ---- block gather ----------------------------------------------------------
-// Stage the non-empty segments among [s0, s0+n) of row r: sd_ptr[k] points
-// at the segment minus its start offset in the concatenation (so product q
-// of segment k is sd_ptr[k][q]), sd_end[k] is its inclusive end.  Returns the
-// number of products; *ns = number of staged segments.  Ends with a barrier.
+// Stage segments [s0, s0+n) of row r: sd_ptr[k] points at the segment minus
+// its start offset in the batch's concatenation (so product q of segment k
+// is sd_ptr[k][q]), sd_end[k] is its exclusive end.  Descriptor mode: a
+// plain copy of the precomputed descriptors (non-empty, prefix ends).
+// Returns the number of products in the batch; ends with a barrier.
 template <int THREADS>
 __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint32_t s0, uint32_t n,
-                                                   const idx_t** sd_ptr, uint32_t* sd_end, uint64_t* s_scan,
-                                                   uint32_t* ns) {
-    const uint32_t per = (n + THREADS - 1) / THREADS;
-    const uint32_t b = threadIdx.x * per, e = min(b + per, n);
-    uint64_t acc = 0;  // (non-empty count << 32) | product count
-#pragma unroll 1
-    for (uint32_t i = b; i < e; ++i) {
-        uint32_t len;
-        get_seg(s, r, s0 + i, len);
-        if (len) acc += (1ull << 32) + len;
-    }
-    uint64_t tot;
-    const uint64_t ex = block_exclusive_scan<uint64_t>(acc, s_scan, &tot);
-    uint32_t k = uint32_t(ex >> 32), run = uint32_t(ex);
-#pragma unroll 1
-    for (uint32_t i = b; i < e; ++i) {
-        uint32_t len;
-        const idx_t* p = get_seg(s, r, s0 + i, len);
-        if (len) {
-            sd_ptr[k] = p - run;
-            run += len;
-            sd_end[k] = run;
-            ++k;
+                                                   const idx_t** sd_ptr, uint32_t* sd_end) {
+    if (s.kind == 1) {  // one segment
+        if (threadIdx.x == 0) {
+            const off_t64 b = s.lrp[r];
+            sd_ptr[0] = s.lst + b;
+            sd_end[0] = uint32_t(s.lrp[r + 1] - b);
         }
+        __syncthreads();
+        return sd_end[0];
+    }
+    const uint4* d = s.desc + (s.dbase[r] + r + s0);
+    const uint32_t base = s0 ? s.desc[s.dbase[r] + r + s0 - 1].w : 0u;
+#pragma unroll 1
+    for (uint32_t i = threadIdx.x; i < n; i += THREADS) {
+        const uint4 e = d[i];
+        const idx_t* p = reinterpret_cast<const idx_t*>((uint64_t(e.y) << 32) | e.x);
+        const uint32_t end = e.w - base;
+        sd_ptr[i] = p - (end - e.z);
+        sd_end[i] = end;
     }
     __syncthreads();
-    *ns = uint32_t(tot >> 32);
-    return uint32_t(tot);
+    return d[n - 1].w - base;
 }
 
 // Call f(c) for every product of row r.  Thread t takes U consecutive
@@ -202,11 +183,11 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
 // Ends with a barrier.
 template <int THREADS, int U, typename F>
 __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, const idx_t** sd_ptr,
-                                               uint32_t* sd_end, uint32_t batch, uint64_t* s_scan, F&& f) {
+                                               uint32_t* sd_end, uint32_t batch, F&& f) {
     const uint32_t nseg = num_segs(s, r);
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
-        uint32_t ns;
-        const uint32_t total = stage_segments<THREADS>(s, r, s0, min(batch, nseg - s0), sd_ptr, sd_end, s_scan, &ns);
+        const uint32_t ns = min(batch, nseg - s0);
+        const uint32_t total = stage_segments<THREADS>(s, r, s0, ns, sd_ptr, sd_end);
 #ifdef SPBLA_PROBE
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
@@ -407,25 +388,33 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     uint32_t* poff = obcnt + OBCAP;  // [MP] output offset of each bucket pair
     uint32_t* wbuf = reinterpret_cast<uint32_t*>(sd_ptr);
     static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0, "hash bin layout");
-    __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_wt[KP][NW], s_total;
-    __shared__ uint32_t s_item, s_flag, s_novf, s_nob, s_pool;
+    __shared__ uint32_t s_wt[KP][NW];
+    __shared__ uint32_t s_item[2], s_flag, s_novf, s_nob, s_pool;
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
+    // the table is kept clean between rows (all slots 0xFFFF, counters 0):
+    // every row restores what it dirtied before the end-of-row barrier
+#pragma unroll 1
+    for (uint32_t i = threadIdx.x; i < 8 * MAXB; i += THREADS) tabw[i] = 0xFFFFFFFFu;
+#pragma unroll 1
+    for (uint32_t i = threadIdx.x; i < MAXB; i += THREADS) bcnt[i] = 0u;
+    if (threadIdx.x == 0) s_item[0] = lo_i + atomicAdd(work, 1u);
+    __syncthreads();
     PROBE_DECL
-    for (;;) {
+#pragma unroll 1
+    for (uint32_t it = 0;; ++it) {
+        // the next row is claimed while this one runs: one barrier per row boundary
+        const uint32_t item = s_item[it & 1];
+        if (item >= hi_i) break;
         if (threadIdx.x == 0) {
-            s_item = lo_i + atomicAdd(work, 1u);
+            s_item[(it + 1) & 1] = lo_i + atomicAdd(work, 1u);
             s_flag = 0;
             s_novf = 0;
             s_nob = 0;
             s_pool = 0;
         }
-        __syncthreads();
-        const uint32_t item = s_item;
-        if (item >= hi_i) break;
         PROBE(0);
         const idx_t r = rows[item];
         const uint32_t u = uint32_t(ub[r]);
@@ -441,19 +430,24 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         const uint64_t nbw = (span + 65534) / 65535;
         const uint32_t nb =
             (uint32_t(min(max(max(uint64_t((u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB))) + 1) & ~1u;
+        const uint32_t np = nb / 2;
         const uint64_t words = (span + 31) >> 5;
         idx_t* out = scratch + soff[r];
         if (words <= 9ull * nb) {  // the span bitmap is no larger than the table
             const uint32_t nw = uint32_t(words);
-            fill_words(bmw, nw, 0u, THREADS);
+#pragma unroll 1
+            for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = 0u;
             __syncthreads();
-            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, [&](idx_t c) {
                 const uint32_t d = c - clo;
                 atomicOr(&bmw[d >> 5], 1u << (d & 31));
             });
             const uint32_t n = emit_bitmap<NW>(bmw, nw, clo, out, s_w);
             if (threadIdx.x == 0) counts[r] = n;
-            continue;  // emit_bitmap ends with a barrier
+#pragma unroll 1
+            for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = i < 8 * MAXB ? 0xFFFFFFFFu : 0u;
+            __syncthreads();
+            continue;
         }
         PROBE(1);
         if (nbw > MAXB) {  // span too wide for 16-bit offsets in this table
@@ -467,15 +461,8 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         const uint32_t W = uint32_t((span + nb - 1) / nb);
         const uint32_t l = (32 - __clz(W - 1)) - 3;
         const uint32_t M = uint32_t(((uint64_t(1) << (32 + l)) + W - 1) / W);
-        const uint32_t np = nb / 2;
-#pragma unroll 1
-        for (uint32_t sl = 0; sl < kSlots; ++sl)
-#pragma unroll 1
-            for (uint32_t i = threadIdx.x; i < np; i += THREADS) tabw[sl * MP + i] = 0xFFFFFFFFu;
-        fill_words(bcnt, nb, 0u, THREADS);
-        __syncthreads();
         PROBE(2);
-        block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+        block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, [&](idx_t c) {
             const uint32_t d = c - clo;
             const uint32_t b = __umulhi(d, M) >> l;
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
@@ -486,57 +473,50 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 if (i < OVCAP) ovl[i] = c; else s_flag = 1;
             }
         });
-        if (s_flag) {  // overflow list full: hand the row to the bitmap bin
-            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
-            __syncthreads();  // everyone has read s_flag / s_item before reuse
-            continue;
-        }
         PROBE(4);
-        // ---- pass A: sort each owned bucket pair in 16x2 SIMD ----------------
-        // (rolled loops from here on: the kernel must stay small for the I-cache)
-        // bcnt[b] becomes the bucket's distinct count, or kOvfFlag | list index
+        bool fallback = s_flag != 0;  // overflow list full: the row goes to the bitmap bin
+        if (!fallback) {
+            // ---- pass A: sort each owned bucket pair in 16x2 SIMD ----------------
+            // bcnt[b] becomes the bucket's distinct count, or kOvfFlag | list index
 #pragma unroll 1
-        for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
-            const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
-            uint32_t keep = 0xFFFFFFFFu;  // lanes of an overflowed bucket are masked out of the sort
-            uint2 res;
-            if (nn.x > kSlots) {
-                const uint32_t j = atomicAdd(&s_nob, 1u);
-                if (j < OBCAP) obl[j] = 2 * m; else s_flag = 1;
-                res.x = kOvfFlag | j;
-                keep &= 0xFFFF0000u;
+            for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
+                const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+                uint32_t keep = 0xFFFFFFFFu;  // lanes of an overflowed bucket are masked out of the sort
+                uint2 res;
+                if (nn.x > kSlots) {
+                    const uint32_t j = atomicAdd(&s_nob, 1u);
+                    if (j < OBCAP) obl[j] = 2 * m; else s_flag = 1;
+                    res.x = kOvfFlag | j;
+                    keep &= 0xFFFF0000u;
+                }
+                if (nn.y > kSlots) {
+                    const uint32_t j = atomicAdd(&s_nob, 1u);
+                    if (j < OBCAP) obl[j] = 2 * m + 1; else s_flag = 1;
+                    res.y = kOvfFlag | j;
+                    keep &= 0x0000FFFFu;
+                }
+                uint32_t x[16];
+#pragma unroll
+                for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m] | ~keep;
+                sort16x2(x);
+                // adjacent equal pairs: max(x_i, x_{i-1}+1) - x_i is 1 iff x_i == x_{i-1}
+                // (an empty 0xFFFF predecessor wraps to 0 and counts nothing); the
+                // per-half differences are >= 0, so a plain 32-bit sum keeps them apart
+                uint32_t dsum = 0;
+#pragma unroll
+                for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
+                if (nn.x <= kSlots) res.x = nn.x - (dsum & 0xFFFFu);
+                if (nn.y <= kSlots) res.y = nn.y - (dsum >> 16);
+                reinterpret_cast<uint2*>(bcnt)[m] = res;
+                // an overflowed bucket keeps its raw slots for the overflow pass
+#pragma unroll
+                for (int sl = 0; sl < 16; ++sl) tabw[sl * MP + m] = (x[sl] & keep) | (tabw[sl * MP + m] & ~keep);
             }
-            if (nn.y > kSlots) {
-                const uint32_t j = atomicAdd(&s_nob, 1u);
-                if (j < OBCAP) obl[j] = 2 * m + 1; else s_flag = 1;
-                res.y = kOvfFlag | j;
-                keep &= 0x0000FFFFu;
-            }
-            uint32_t x[16];
-#pragma unroll
-            for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m] | ~keep;
-            sort16x2(x);
-            // adjacent equal pairs: max(x_i, x_{i-1}+1) - x_i is 1 iff x_i == x_{i-1}
-            // (an empty 0xFFFF predecessor wraps to 0 and counts nothing); the
-            // per-half differences are >= 0, so a plain 32-bit sum keeps them apart
-            uint32_t dsum = 0;
-#pragma unroll
-            for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
-            if (nn.x <= kSlots) res.x = nn.x - (dsum & 0xFFFFu);
-            if (nn.y <= kSlots) res.y = nn.y - (dsum >> 16);
-            reinterpret_cast<uint2*>(bcnt)[m] = res;
-            // an overflowed bucket keeps its raw slots for the overflow pass
-#pragma unroll
-            for (int sl = 0; sl < 16; ++sl) tabw[sl * MP + m] = (x[sl] & keep) | (tabw[sl * MP + m] & ~keep);
-        }
-        __syncthreads();
-        const uint32_t nob = s_nob;
-        if (s_flag) {
-            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
             __syncthreads();
-            continue;
+            fallback = s_flag != 0;
         }
-        if (nob) {
+        const uint32_t nob = s_nob;
+        if (!fallback && nob) {
             // ---- overflow buckets: one warp each, <= 32 values sorted across lanes
             const uint32_t novf = s_novf;
             uint32_t* wb = wbuf + wib * 32;
@@ -580,80 +560,83 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 if (lane == 0) obcnt[j] = (mcnt << 16) | off;
             }
             __syncthreads();
-            if (s_flag) {
-                if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
-                __syncthreads();
-                continue;
-            }
+            fallback = s_flag != 0;
         }
-        PROBE(5);
-        // ---- multi-scan: output offset of every owned pair -> poff[m] ----------
-        auto bucket_count = [&](uint32_t x) { return (x & kOvfFlag) ? obcnt[x & ~kOvfFlag] >> 16 : x; };
-        uint32_t cpair[KP], inc[KP];
+        if (fallback) {
+            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+        } else {
+            PROBE(5);
+            // ---- multi-scan: output offset of every owned pair (one barrier) -----
+            auto bucket_count = [&](uint32_t x) { return (x & kOvfFlag) ? obcnt[x & ~kOvfFlag] >> 16 : x; };
+            uint32_t cpair[KP], inc[KP];
 #pragma unroll
-        for (uint32_t i = 0; i < KP; ++i) {
-            const uint32_t m = threadIdx.x + i * THREADS;
-            cpair[i] = 0;
-            if (m < np) {
-                const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
-                cpair[i] = bucket_count(nn.x) + bucket_count(nn.y);
+            for (uint32_t i = 0; i < KP; ++i) {
+                const uint32_t m = threadIdx.x + i * THREADS;
+                cpair[i] = 0;
+                if (m < np) {
+                    const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+                    cpair[i] = bucket_count(nn.x) + bucket_count(nn.y);
+                }
+                inc[i] = warp_inclusive_scan(cpair[i]);
+                if (lane == 31) s_wt[i][wib] = inc[i];
             }
-            inc[i] = warp_inclusive_scan(cpair[i]);
-            if (lane == 31) s_wt[i][wib] = inc[i];
-        }
-        __syncthreads();
-        if (wib == 0) {
+            __syncthreads();
+            // every warp scans the (round, warp) totals itself
             uint32_t carry = 0;
 #pragma unroll
             for (uint32_t i = 0; i < KP; ++i) {
                 const uint32_t v = lane < NW ? s_wt[i][lane] : 0u;
                 const uint32_t vi = warp_inclusive_scan(v);
-                if (lane < NW) s_wt[i][lane] = carry + vi - v;
+                const uint32_t wpre = __shfl_sync(FULL, vi - v, wib);  // (all lanes: not inside the branch)
+                const uint32_t m = threadIdx.x + i * THREADS;
+                if (m < np) poff[m] = carry + wpre + inc[i] - cpair[i];
                 carry += __shfl_sync(FULL, vi, 31);
             }
-            if (lane == 0) s_total = carry;
-        }
-        __syncthreads();
+            if (threadIdx.x == 0) counts[r] = carry;
+            PROBE(6);
+            // ---- pass B: stream the sorted pairs, skipping adjacent duplicates -----
+            // (each thread reads back only its own poff entries: no barrier needed)
+#pragma unroll 1
+            for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
+                idx_t* o = out + poff[m];
+                const idx_t base0 = clo + 2 * m * W, base1 = base0 + W;
+                const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+                uint32_t x[16];
 #pragma unroll
-        for (uint32_t i = 0; i < KP; ++i) {
-            const uint32_t m = threadIdx.x + i * THREADS;
-            if (m < np) poff[m] = s_wt[i][wib] + inc[i] - cpair[i];
+                for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m];
+                uint32_t pos = 0, prev = 0xFFFFu;
+#pragma unroll
+                for (int sl = 0; sl < 16; ++sl) {
+                    const uint32_t v = x[sl] & 0xFFFFu;
+                    emit_if(o, pos, base0, v, prev);
+                    prev = v;
+                }
+                if (nn.x & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
+                    const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                    for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base0 + pool[off + j - kSlots];
+                }
+                prev = 0xFFFFu;
+#pragma unroll
+                for (int sl = 0; sl < 16; ++sl) {
+                    const uint32_t v = x[sl] >> 16;
+                    emit_if(o, pos, base1, v, prev);
+                    prev = v;
+                }
+                if (nn.y & kOvfFlag) {
+                    const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                    for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base1 + pool[off + j - kSlots];
+                }
+            }
         }
-        PROBE(6);
-        // ---- pass B: stream the sorted pairs, skipping adjacent duplicates -----
-        // (each thread reads back only its own poff entries: no barrier needed)
+        // ---- restore the pairs this row dirtied (each thread its own) ---------
+        // (pass A / B touched only owned pairs; inserts and the overflow pass
+        // touched pairs < np, all of which have an owner)
 #pragma unroll 1
         for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
-            idx_t* o = out + poff[m];
-            const idx_t base0 = clo + 2 * m * W, base1 = base0 + W;
-            const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
-            uint32_t x[16];
 #pragma unroll
-            for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m];
-            uint32_t pos = 0, prev = 0xFFFFu;
-#pragma unroll
-            for (int sl = 0; sl < 16; ++sl) {
-                const uint32_t v = x[sl] & 0xFFFFu;
-                emit_if(o, pos, base0, v, prev);
-                prev = v;
-            }
-            if (nn.x & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
-                const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
-                for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base0 + pool[off + j - kSlots];
-            }
-            prev = 0xFFFFu;
-#pragma unroll
-            for (int sl = 0; sl < 16; ++sl) {
-                const uint32_t v = x[sl] >> 16;
-                emit_if(o, pos, base1, v, prev);
-                prev = v;
-            }
-            if (nn.y & kOvfFlag) {
-                const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
-                for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base1 + pool[off + j - kSlots];
-            }
+            for (int sl = 0; sl < 16; ++sl) tabw[sl * MP + m] = 0xFFFFFFFFu;
+            reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
         }
-        if (threadIdx.x == 0) counts[r] = s_total;
         __syncthreads();
         PROBE(7);
         PROBE_PRINT("hash", u, num_segs(src, r));
@@ -701,7 +684,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         for (uint32_t w = 0; w < nwin; ++w) {
             const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseBits;
             const uint64_t whi = min(wlo + kDenseBits, uint64_t(chi) + 1);
-            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, s_scan, [&](idx_t c) {
+            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, [&](idx_t c) {
                 if (c >= wlo && c < whi) {
                     const uint32_t d = uint32_t(c - wlo);
                     const uint32_t bit = 1u << (d & 31);
