@@ -8,10 +8,11 @@ import paper_conf_ipps_orachevkkg21_b200 as sp
 scale = int(sys.argv[1]) if len(sys.argv) > 1 else 20
 ef = int(sys.argv[2]) if len(sys.argv) > 2 else 16
 a, b, c = (float(x) for x in (sys.argv[3:6] if len(sys.argv) > 5 else (0.45, 0.22, 0.22)))
+seed = int(sys.argv[6]) if len(sys.argv) > 6 else 1
 sp.Initialize(0)
 n = 1 << scale
 t = time.time()
-r, cc = spgen.rmat_pairs(scale, ef, a, b, c, seed=1, device="cuda")
+r, cc = spgen.rmat_pairs(scale, ef, a, b, c, seed=seed, device="cuda")
 torch.cuda.synchronize(); print("gen", time.time() - t, flush=True)
 t = time.time()
 A = sp.Matrix.from_pairs(n, n, r, cc)
