@@ -273,7 +273,7 @@ def main():
     log(f"[rank {rank}] step ms: {[round(x, 2) for x in step_ms]}")
     launches = sp.launch_count()
     ktimes = {k: sp.kernel_timing(k) for k in
-              ("mxm_ub", "warp_bins", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "compact")}
+              ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "compact")}
     sp.set_kernel_timing(False)
     peak_mem = sp.memory_stats()[1]
     red_dev = "cpu" if world > 1 and dist.get_backend() == "gloo" else "cuda"
@@ -294,15 +294,15 @@ def main():
     thr = sp.engine_thresholds()
     peak_gbs, peak_src = load_peaks()
     roof = None
-    dom = max(("warp_bins", "H1", "H2", "H3", "H4", "H5", "H6", "dense"), key=lambda k: ktimes[k][0])
+    dom = max(("warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense"), key=lambda k: ktimes[k][0])
     dms, dn = ktimes[dom]
     if dn:
         rp_a, ci_a = A.device_tensors()
         crp, _ = C.device_tensors()
         lens_a = (rp_a[1:] - rp_a[:-1])
         outs = (crp[1:] - crp[:-1])
-        bins = {"warp_bins": (0, thr[4]), "dense": (thr[10], 1 << 62)}
-        bins.update({f"H{i}": (thr[3 + i], thr[4 + i]) for i in range(1, 7)})
+        bins = {"warp_bins": (0, thr[3]), "dense": (thr[10], 1 << 62)}
+        bins.update({f"H{i}": (thr[3 + i], thr[4 + i]) for i in range(0, 7)})
         lo_hi = bins[dom]
         sel = (ub > lo_hi[0]) & (ub <= lo_hi[1])
         seg = int(lens_a[sel].sum())

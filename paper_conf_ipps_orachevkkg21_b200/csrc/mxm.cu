@@ -17,9 +17,20 @@ namespace {
 
 constexpr int kGroup = 8;
 
+// Column span of every B row: bspan[k] = (B[k][0], B[k][last]) (rows are
+// sorted), (0xFFFFFFFF, 0) for an empty row.  8 B per row: the upper-bound
+// pass then reads one L2-resident word per A entry instead of two scattered
+// colidx sectors.
+__global__ void row_span_kernel(CsrView B, uint2* __restrict__ bspan) {
+    for (size_t k = blockIdx.x * size_t(blockDim.x) + threadIdx.x; k < B.nrows; k += size_t(gridDim.x) * blockDim.x) {
+        const off_t64 x = B.rowptr[k], y = B.rowptr[k + 1];
+        bspan[k] = y > x ? make_uint2(B.colidx[x], B.colidx[y - 1]) : make_uint2(0xFFFFFFFFu, 0u);
+    }
+}
+
 __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
-                              const off_t64* __restrict__ crp, const idx_t* __restrict__ cci,
-                              uint64_t* __restrict__ ub, uint2* __restrict__ range,
+                              const uint2* __restrict__ bspan, const off_t64* __restrict__ crp,
+                              const idx_t* __restrict__ cci, uint64_t* __restrict__ ub, uint2* __restrict__ range,
                               uint4* __restrict__ desc, uint32_t* __restrict__ nseg) {
     const unsigned lane = threadIdx.x & 31, g = lane & (kGroup - 1);
     const unsigned gshift = lane & ~(kGroup - 1);  // first lane of this row's group
@@ -32,6 +43,7 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
         uint64_t s = 0;
         off_t64 b = 0, e = 0;
         uint32_t cn = 0, cl = 0;  // running non-empty count / product prefix of the row
+        idx_t lo = 0xFFFFFFFFu, hi = 0;
         uint4* drow = nullptr;
         if (valid) {
             b = A.rowptr[r];
@@ -44,10 +56,12 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
                     if (g == 0) {
                         const uint64_t ptr = reinterpret_cast<uint64_t>(cci + cb);
                         drow[0] = make_uint4(uint32_t(ptr), uint32_t(ptr >> 32), lc, lc);
+                        s = lc;
+                        lo = cci[cb];
+                        hi = cci[cb + lc - 1];
                     }
                     cn = 1;
                     cl = lc;
-                    s = g == 0 ? lc : 0;
                 }
             }
         }
@@ -59,8 +73,11 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
             if (valid && p < e) {
                 const idx_t k = A.colidx[p];
                 const off_t64 x = brp[k], y = brp[k + 1];
+                const uint2 sp = bspan[k];  // (0xFFFFFFFF, 0) when empty: neutral
                 len = uint32_t(y - x);
                 ptr = reinterpret_cast<uint64_t>(bci + x);
+                lo = min(lo, sp.x);
+                hi = max(hi, sp.y);
             }
             s += len;
             // compacted position and inclusive length prefix inside the group
@@ -75,35 +92,18 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
             cn += __popc(m);
             cl += __shfl_sync(0xffffffffu, inc, kGroup - 1, kGroup);
         }
-#pragma unroll
-        for (int d = kGroup / 2; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d, kGroup);
-        // column span of the row (segments are sorted: first / last entries),
-        // used by the hash and bitmap bins of the row engine
-        const bool need = valid && s > kRangeMinUb;
-        idx_t lo = 0xFFFFFFFFu, hi = 0;
-        if (need) {
-            for (off_t64 p = b + g; p < e; p += kGroup) {
-                idx_t k = A.colidx[p];
-                off_t64 x = brp[k], y = brp[k + 1];
-                if (y > x) {
-                    lo = min(lo, bci[x]);
-                    hi = max(hi, bci[y - 1]);
-                }
-            }
-            if (g == 0 && crp && crp[r + 1] > crp[r]) {
-                lo = min(lo, cci[crp[r]]);
-                hi = max(hi, cci[crp[r + 1] - 1]);
-            }
-        }
+        // row totals and column span (segments are sorted: first / last
+        // entries), the span used by the hash and bitmap bins of the engine
 #pragma unroll
         for (int d = kGroup / 2; d > 0; d >>= 1) {
+            s += __shfl_xor_sync(0xffffffffu, s, d, kGroup);
             lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, d, kGroup));
             hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, d, kGroup));
         }
         if (valid && g == 0) {
             ub[r] = s;
             nseg[r] = cn;
-            if (need) range[r] = make_uint2(lo, hi);
+            if (s > kRangeMinUb) range[r] = make_uint2(lo, hi);
         }
     }
 }
@@ -130,8 +130,14 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
                                                        uint64_t(ctx().num_sms) * 16);
     const off_t64* crp = accumulate ? C->rowptr : nullptr;
+    DevBuf<uint2> bspan(B->nrows);
     int tk = ktime_begin("mxm_ub", ctx().stream);
-    mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, crp,
+    if (B->nrows) {
+        const unsigned gs = (unsigned)std::min<uint64_t>(ceil_div(B->nrows, 256), uint64_t(ctx().num_sms) * 16);
+        row_span_kernel<<<gs, 256, 0, ctx().stream>>>(view(B), bspan.p);
+        count_launch();
+    }
+    mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, bspan.p, crp,
                                                   accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p, nseg.p);
     ktime_end(tk);
     count_launch();

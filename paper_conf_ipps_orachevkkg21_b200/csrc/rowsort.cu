@@ -66,12 +66,12 @@ __shared__ unsigned long long s_probe_ext[12];
 #endif
 constexpr int kNumBins = 13;
 enum {
-    BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_W16,
+    BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_H0,
     BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_H6, BIN_DENSE = 12
 };
-constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 512
+constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 // hash bins: ub limits (each sized so its tables fit the residency below)
-constexpr uint64_t kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480, kH6 = 40960;
+constexpr uint64_t kH0 = 512, kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480, kH6 = 40960;
 constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
@@ -80,8 +80,8 @@ __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub <= 32) return BIN_W1;
     if (ub <= 64) return BIN_W2;
     if (ub <= 128) return BIN_W4;
-    if (ub <= 256) return BIN_W8;
-    if (ub <= kWarpMaxUb) return BIN_W16;
+    if (ub <= kWarpMaxUb) return BIN_W8;
+    if (ub <= kH0) return BIN_H0;
     if (ub <= kH1) return BIN_H1;
     if (ub <= kH2) return BIN_H2;
     if (ub <= kH3) return BIN_H3;
@@ -147,10 +147,14 @@ __device__ __forceinline__ uint32_t warp_flat(const idx_t* p, uint32_t len, F&& 
 // its start offset in the batch's concatenation (so product q of segment k
 // is sd_ptr[k][q]), sd_end[k] is its exclusive end.  Descriptor mode: a
 // plain copy of the precomputed descriptors (non-empty, prefix ends).
+// sd_first (nullable): sd_first[j] = the segment holding product j << kFirstShift,
+// written by that segment (each multiple of 2^kFirstShift lies in exactly one
+// non-empty segment); replaces the binary search of the gather.
 // Returns the number of products in the batch; ends with a barrier.
+constexpr uint32_t kFirstShift = 6;
 template <int THREADS>
 __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint32_t s0, uint32_t n,
-                                                   const idx_t** sd_ptr, uint32_t* sd_end) {
+                                                   const idx_t** sd_ptr, uint32_t* sd_end, uint32_t* sd_first) {
     if (s.kind == 1) {  // one segment
         if (threadIdx.x == 0) {
             const off_t64 b = s.lrp[r];
@@ -166,9 +170,14 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
     for (uint32_t i = threadIdx.x; i < n; i += THREADS) {
         const uint4 e = d[i];
         const idx_t* p = reinterpret_cast<const idx_t*>((uint64_t(e.y) << 32) | e.x);
-        const uint32_t end = e.w - base;
-        sd_ptr[i] = p - (end - e.z);
+        const uint32_t end = e.w - base, start = end - e.z;
+        sd_ptr[i] = p - start;
         sd_end[i] = end;
+        if (sd_first) {
+#pragma unroll 1
+            for (uint32_t j = (start + (1u << kFirstShift) - 1) >> kFirstShift; (j << kFirstShift) < end; ++j)
+                sd_first[j] = i;
+        }
     }
     __syncthreads();
     return d[n - 1].w - base;
@@ -176,29 +185,39 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
 
 // Call f(c) for every product of row r.  Thread t takes U consecutive
 // products q0 = (t + i*THREADS)*U .. q0+U-1 of the concatenated segments:
-// one binary search over the staged segment ends for q0, then a linear
-// advance (segments average tens of products, so a run rarely crosses more
-// than one boundary); the U loads are issued before any insert.  A warp
-// covers 32*U consecutive products, i.e. a few sectors of each B row.
-// Ends with a barrier.
+// the segment holding q0 comes from the sd_first table plus a short linear
+// advance (binary search when there is no table), then a linear advance
+// inside the run (segments average tens of products, so a run rarely
+// crosses more than one boundary); the U loads are issued before any
+// insert.  A warp covers 32*U consecutive products, i.e. a few sectors of
+// each B row.  Ends with a barrier.
 template <int THREADS, int U, typename F>
 __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, const idx_t** sd_ptr,
-                                               uint32_t* sd_end, uint32_t batch, F&& f) {
+                                               uint32_t* sd_end, uint32_t* sd_first, uint32_t batch, F&& f) {
     const uint32_t nseg = num_segs(s, r);
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
         const uint32_t ns = min(batch, nseg - s0);
-        const uint32_t total = stage_segments<THREADS>(s, r, s0, ns, sd_ptr, sd_end);
+        const uint32_t total = stage_segments<THREADS>(s, r, s0, ns, sd_ptr, sd_end, sd_first);
 #ifdef SPBLA_PROBE
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
         for (uint32_t q0 = threadIdx.x * U; q0 < total; q0 += THREADS * U) {
-            uint32_t lo = 0, hi = ns - 1;  // first segment whose end exceeds q0
-            while (lo < hi) {
-                const uint32_t mid = (lo + hi) >> 1;
-                if (sd_end[mid] <= q0) lo = mid + 1; else hi = mid;
+            uint32_t k;
+            if (s.kind == 1) {
+                k = 0;
+            } else if (sd_first) {
+                k = sd_first[q0 >> kFirstShift];
+                while (sd_end[k] <= q0) ++k;
+            } else {
+                uint32_t lo = 0, hi = ns - 1;  // first segment whose end exceeds q0
+                while (lo < hi) {
+                    const uint32_t mid = (lo + hi) >> 1;
+                    if (sd_end[mid] <= q0) lo = mid + 1; else hi = mid;
+                }
+                k = lo;
             }
-            uint32_t k = lo, end = sd_end[lo];
-            const idx_t* p = sd_ptr[lo];
+            uint32_t end = sd_end[k];
+            const idx_t* p = sd_ptr[k];
             idx_t v[U];
             // consecutive products cross at most one boundary (segments are
             // non-empty), so each step is a single predicated advance
@@ -341,28 +360,21 @@ __device__ __forceinline__ uint32_t vadd2(uint32_t a, uint32_t b) {  // per-16-b
     asm("add.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
     return r;
 }
-// o[pos] = base + v and pos += 1 if v is a valid slot (!= 0xFFFF) distinct from prev
-__device__ __forceinline__ void emit_if(idx_t* o, uint32_t& pos, uint32_t base, uint32_t v, uint32_t prev) {
-    asm volatile(
-        "{\n\t.reg .pred q;\n\t.reg .u64 a;\n\t.reg .u32 x;\n\t"
-        "setp.ne.u32 q, %2, %3;\n\t"
-        "setp.ne.and.u32 q, %2, 65535, q;\n\t"
-        "mad.wide.u32 a, %0, 4, %4;\n\t"
-        "add.u32 x, %1, %2;\n\t"
-        "@q st.global.u32 [a], x;\n\t"
-        "@q add.u32 %0, %0, 1;\n\t}"
-        : "+r"(pos)
-        : "r"(base), "r"(v), "r"(prev), "l"(o)
-        : "memory");
-}
 constexpr uint32_t kOvfFlag = 0x80000000u;
 constexpr uint32_t kSlots = 16;
 
 template <int E>
 __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]);
 
-// dynamic smem: tab16[16*MAXB] | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | ovl[OVCAP] |
-//               pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | poff[MAXB/2]
+// Pair stride of the slot-major table: MPP = 2 (mod 32), so slot s of pair m
+// sits in bank 2s + m (mod 32): the per-thread pass A (lanes = consecutive
+// pairs, one slot) and the warp-cooperative pass B (lanes = 16 slots x 2
+// consecutive pairs) are both conflict-free.
+__host__ __device__ constexpr uint32_t pair_stride(uint32_t mp) { return ((mp + 29) / 32) * 32 + 2; }
+__host__ __device__ constexpr uint32_t first_entries(uint64_t maxub) { return uint32_t((maxub >> kFirstShift) + 1); }
+
+// dynamic smem: tabw[16*MPP] | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | sd_first[NF] |
+//               ovl[OVCAP] | pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | poff[MAXB/2]
 // (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
 // which are dead once the products are inserted: BATCH * 3 >= THREADS)
 template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU>
@@ -373,21 +385,25 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
     constexpr int NW = THREADS / 32;
     constexpr uint32_t MP = MAXB / 2;                      // bucket pairs
+    constexpr uint32_t MPP = pair_stride(MP);              // padded pair stride of the table
+    constexpr uint32_t TABW = 16 * MPP;                    // table words
     constexpr uint32_t KP = (MP + THREADS - 1) / THREADS;  // pairs per thread
+    constexpr uint32_t NF = first_entries(uint64_t(MAXB) * 8);
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    uint32_t* tabw = reinterpret_cast<uint32_t*>(smem_raw);  // word s*MP + m = slot s of pair m
+    uint32_t* tabw = reinterpret_cast<uint32_t*>(smem_raw);  // word s*MPP + m = slot s of pair m
     uint16_t* tab16 = reinterpret_cast<uint16_t*>(smem_raw);
-    uint32_t* bmw = tabw;  // bitmap-mode view: MAXB * 9 words
-    uint32_t* bcnt = tabw + 8 * MAXB;
+    uint32_t* bmw = tabw;  // bitmap-mode view: TABW + MAXB words
+    uint32_t* bcnt = tabw + TABW;
     const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(bcnt + MAXB);
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(sd_ptr + BATCH);
-    idx_t* ovl = sd_end + BATCH;
+    uint32_t* sd_first = sd_end + BATCH;
+    idx_t* ovl = sd_first + NF;
     uint16_t* pool = reinterpret_cast<uint16_t*>(ovl + OVCAP);
     uint32_t* obl = reinterpret_cast<uint32_t*>(pool + OVCAP);
     uint32_t* obcnt = obl + OBCAP;
     uint32_t* poff = obcnt + OBCAP;  // [MP] output offset of each bucket pair
     uint32_t* wbuf = reinterpret_cast<uint32_t*>(sd_ptr);
-    static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0, "hash bin layout");
+    static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0 && MP % 32 == 0, "hash bin layout");
     __shared__ uint32_t s_w[33];
     __shared__ uint32_t s_wt[KP][NW];
     __shared__ uint32_t s_item[2], s_flag, s_novf, s_nob, s_pool;
@@ -397,7 +413,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     // the table is kept clean between rows (all slots 0xFFFF, counters 0):
     // every row restores what it dirtied before the end-of-row barrier
 #pragma unroll 1
-    for (uint32_t i = threadIdx.x; i < 8 * MAXB; i += THREADS) tabw[i] = 0xFFFFFFFFu;
+    for (uint32_t i = threadIdx.x; i < TABW; i += THREADS) tabw[i] = 0xFFFFFFFFu;
 #pragma unroll 1
     for (uint32_t i = threadIdx.x; i < MAXB; i += THREADS) bcnt[i] = 0u;
     if (threadIdx.x == 0) s_item[0] = lo_i + atomicAdd(work, 1u);
@@ -438,14 +454,14 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
 #pragma unroll 1
             for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = 0u;
             __syncthreads();
-            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, [&](idx_t c) {
+            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, sd_first, BATCH, [&](idx_t c) {
                 const uint32_t d = c - clo;
                 atomicOr(&bmw[d >> 5], 1u << (d & 31));
             });
             const uint32_t n = emit_bitmap<NW>(bmw, nw, clo, out, s_w);
             if (threadIdx.x == 0) counts[r] = n;
 #pragma unroll 1
-            for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = i < 8 * MAXB ? 0xFFFFFFFFu : 0u;
+            for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = i < TABW ? 0xFFFFFFFFu : 0u;
             __syncthreads();
             continue;
         }
@@ -462,12 +478,12 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         const uint32_t l = (32 - __clz(W - 1)) - 3;
         const uint32_t M = uint32_t(((uint64_t(1) << (32 + l)) + W - 1) / W);
         PROBE(2);
-        block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, [&](idx_t c) {
+        block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, sd_first, BATCH, [&](idx_t c) {
             const uint32_t d = c - clo;
             const uint32_t b = __umulhi(d, M) >> l;
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
             if (slot < kSlots) {
-                tab16[slot * MAXB + b] = uint16_t(d - b * W);
+                tab16[slot * (2 * MPP) + b] = uint16_t(d - b * W);
             } else {
                 const uint32_t i = atomicAdd(&s_novf, 1u);
                 if (i < OVCAP) ovl[i] = c; else s_flag = 1;
@@ -477,7 +493,10 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         bool fallback = s_flag != 0;  // overflow list full: the row goes to the bitmap bin
         if (!fallback) {
             // ---- pass A: sort each owned bucket pair in 16x2 SIMD ----------------
-            // bcnt[b] becomes the bucket's distinct count, or kOvfFlag | list index
+            // Duplicates are removed in registers (rare: replaced by 0xFFFF and
+            // re-sorted), so every bucket leaves pass A as its distinct values
+            // in slots [0, count) followed by 0xFFFF; bcnt[b] becomes the
+            // bucket's distinct count, or kOvfFlag | list index
 #pragma unroll 1
             for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
                 const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
@@ -497,7 +516,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 }
                 uint32_t x[16];
 #pragma unroll
-                for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m] | ~keep;
+                for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MPP + m] | ~keep;
                 sort16x2(x);
                 // adjacent equal pairs: max(x_i, x_{i-1}+1) - x_i is 1 iff x_i == x_{i-1}
                 // (an empty 0xFFFF predecessor wraps to 0 and counts nothing); the
@@ -505,12 +524,23 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 uint32_t dsum = 0;
 #pragma unroll
                 for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
+                if (dsum) {  // drop the duplicates: mark them empty, sort again
+                    uint32_t prev = x[0];
+#pragma unroll
+                    for (int k2 = 1; k2 < 16; ++k2) {
+                        const uint32_t cur = x[k2];
+                        x[k2] = cur | ((cur & 0xFFFFu) == (prev & 0xFFFFu) ? 0xFFFFu : 0u) |
+                                ((cur >> 16) == (prev >> 16) ? 0xFFFF0000u : 0u);
+                        prev = cur;
+                    }
+                    sort16x2(x);
+                }
                 if (nn.x <= kSlots) res.x = nn.x - (dsum & 0xFFFFu);
                 if (nn.y <= kSlots) res.y = nn.y - (dsum >> 16);
                 reinterpret_cast<uint2*>(bcnt)[m] = res;
                 // an overflowed bucket keeps its raw slots for the overflow pass
 #pragma unroll
-                for (int sl = 0; sl < 16; ++sl) tabw[sl * MP + m] = (x[sl] & keep) | (tabw[sl * MP + m] & ~keep);
+                for (int sl = 0; sl < 16; ++sl) tabw[sl * MPP + m] = (x[sl] & keep) | (tabw[sl * MPP + m] & ~keep);
             }
             __syncthreads();
             fallback = s_flag != 0;
@@ -539,7 +569,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                     continue;
                 }
                 idx_t xv[1];
-                xv[0] = lane < kSlots ? base + tab16[lane * MAXB + b] : (lane < filled ? wb[lane] : kEmpty);
+                xv[0] = lane < kSlots ? base + tab16[lane * (2 * MPP) + b] : (lane < filled ? wb[lane] : kEmpty);
                 __syncwarp();
                 warp_bitonic_sort<1>(xv);
                 const idx_t prev = __shfl_up_sync(FULL, xv[0], 1);
@@ -554,9 +584,9 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 off = __shfl_sync(FULL, off, 0);
                 if (uniq) {
                     const uint16_t o = uint16_t(xv[0] - base);
-                    if (rank < kSlots) tab16[rank * MAXB + b] = o; else pool[off + rank - kSlots] = o;
+                    if (rank < kSlots) tab16[rank * (2 * MPP) + b] = o; else pool[off + rank - kSlots] = o;
                 }
-                if (lane < kSlots && lane >= mcnt) tab16[lane * MAXB + b] = 0xFFFFu;
+                if (lane < kSlots && lane >= mcnt) tab16[lane * (2 * MPP) + b] = 0xFFFFu;
                 if (lane == 0) obcnt[j] = (mcnt << 16) | off;
             }
             __syncthreads();
@@ -593,53 +623,63 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 carry += __shfl_sync(FULL, vi, 31);
             }
             if (threadIdx.x == 0) counts[r] = carry;
+            __syncwarp();
             PROBE(6);
-            // ---- pass B: stream the sorted pairs, skipping adjacent duplicates -----
-            // (each thread reads back only its own poff entries: no barrier needed)
+            // ---- pass B: warp-cooperative emission of the warp's own pairs --------
+            // (pairs 32w + i*THREADS + j were sorted and scanned by this warp's
+            // lanes: no barrier needed).  Lane = (pair m0 + lane/16, slot lane%16):
+            // one word holds slot s of both buckets of the pair; the buckets are
+            // compacted, so slot s of bucket 2m goes to out[poff[m] + s] and of
+            // bucket 2m+1 to out[poff[m] + count(2m) + s].  Each store writes two
+            // runs of <= 16 consecutive columns.  The lane also restores its word.
+            const uint32_t sl = lane & 15u;
 #pragma unroll 1
-            for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
-                idx_t* o = out + poff[m];
-                const idx_t base0 = clo + 2 * m * W, base1 = base0 + W;
-                const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
-                uint32_t x[16];
-#pragma unroll
-                for (int sl = 0; sl < 16; ++sl) x[sl] = tabw[sl * MP + m];
-                uint32_t pos = 0, prev = 0xFFFFu;
-#pragma unroll
-                for (int sl = 0; sl < 16; ++sl) {
-                    const uint32_t v = x[sl] & 0xFFFFu;
-                    emit_if(o, pos, base0, v, prev);
-                    prev = v;
-                }
-                if (nn.x & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
-                    const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
-                    for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base0 + pool[off + j - kSlots];
-                }
-                prev = 0xFFFFu;
-#pragma unroll
-                for (int sl = 0; sl < 16; ++sl) {
-                    const uint32_t v = x[sl] >> 16;
-                    emit_if(o, pos, base1, v, prev);
-                    prev = v;
-                }
-                if (nn.y & kOvfFlag) {
-                    const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
-                    for (uint32_t j = kSlots; j < mc; ++j) o[pos++] = base1 + pool[off + j - kSlots];
+            for (uint32_t i = 0; i < KP; ++i) {
+                const uint32_t mb = i * THREADS + wib * 32;
+#pragma unroll 1
+                for (uint32_t j = 0; j < 32 && mb + j < np; j += 2) {
+                    const uint32_t m = mb + j + (lane >> 4);
+                    if (m < np) {
+                        const uint32_t w = tabw[sl * MPP + m];
+                        tabw[sl * MPP + m] = 0xFFFFFFFFu;
+                        const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+                        const uint32_t c0 = bucket_count(nn.x);
+                        idx_t* o = out + poff[m];
+                        const idx_t base0 = clo + 2 * m * W;
+                        const uint32_t v0 = w & 0xFFFFu, v1 = w >> 16;
+                        if (v0 != 0xFFFFu) o[sl] = base0 + v0;
+                        if (v1 != 0xFFFFu) o[c0 + sl] = base0 + W + v1;
+                        if (sl == 0) {
+                            if ((nn.x | nn.y) & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
+                                if (nn.x & kOvfFlag) {
+                                    const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                                    for (uint32_t q = kSlots; q < mc; ++q) o[q] = base0 + pool[off + q - kSlots];
+                                }
+                                if (nn.y & kOvfFlag) {
+                                    const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                                    for (uint32_t q = kSlots; q < mc; ++q) o[c0 + q] = base0 + W + pool[off + q - kSlots];
+                                }
+                            }
+                            reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
+                        }
+                    }
                 }
             }
+            __syncthreads();
+            PROBE(7);
+            PROBE_PRINT("hash", u, num_segs(src, r));
+            continue;
         }
-        // ---- restore the pairs this row dirtied (each thread its own) ---------
-        // (pass A / B touched only owned pairs; inserts and the overflow pass
+        // ---- fallback: restore the pairs this row dirtied (each thread its own) --
+        // (pass A touched only owned pairs; inserts and the overflow pass
         // touched pairs < np, all of which have an owner)
 #pragma unroll 1
         for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
 #pragma unroll
-            for (int sl = 0; sl < 16; ++sl) tabw[sl * MP + m] = 0xFFFFFFFFu;
+            for (int sl = 0; sl < 16; ++sl) tabw[sl * MPP + m] = 0xFFFFFFFFu;
             reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
         }
         __syncthreads();
-        PROBE(7);
-        PROBE_PRINT("hash", u, num_segs(src, r));
     }
 }
 
@@ -684,7 +724,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         for (uint32_t w = 0; w < nwin; ++w) {
             const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseBits;
             const uint64_t whi = min(wlo + kDenseBits, uint64_t(chi) + 1);
-            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, BATCH, [&](idx_t c) {
+            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, nullptr, BATCH, [&](idx_t c) {
                 if (c >= wlo && c < whi) {
                     const uint32_t d = uint32_t(c - wlo);
                     const uint32_t bit = 1u << (d & 31);
@@ -1056,7 +1096,9 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
 constexpr uint32_t kDBatch = 2048;
 constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, uint32_t ovcap, uint32_t obcap) {
-    return buckets * (8 * sizeof(uint32_t) + sizeof(uint32_t) + sizeof(uint16_t)) + batch * kSegBytes +
+    return size_t(16) * pair_stride(buckets / 2) * sizeof(uint32_t) +          // table
+           buckets * sizeof(uint32_t) + (buckets / 2) * sizeof(uint32_t) +     // counters, pair offsets
+           batch * kSegBytes + first_entries(uint64_t(buckets) * 8) * sizeof(uint32_t) +
            ovcap * (sizeof(idx_t) + sizeof(uint16_t)) + obcap * 2 * sizeof(uint32_t);
 }
 #define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U)                                           \
@@ -1068,13 +1110,15 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
     static_assert(PERSM * T <= 2048, #NAME " threads");
 // <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread>
 // (expected per row at mean load 8 with 16 slots: list ~ub/1500, buckets ~ub/2000)
-HBIN(H1, 128, kH1, 32, 16, 256, 10, 4)
-HBIN(H2, 128, kH2, 32, 16, 256, 10, 4)
-HBIN(H3, 256, kH3, 64, 32, 384, 5, 4)
+HBIN(H0, 32, kH0, 32, 16, 64, 32, 4)
+HBIN(H1, 64, kH1, 32, 16, 128, 20, 4)
+HBIN(H2, 64, kH2, 32, 16, 128, 16, 4)
+HBIN(H3, 128, kH3, 64, 32, 256, 8, 4)
 HBIN(H4, 256, kH4, 64, 32, 256, 4, 8)
 HBIN(H5, 512, kH5, 128, 64, 256, 2, 8)
 HBIN(H6, 1024, kH6, 192, 96, 384, 1, 8)
 #define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U>
+#define HASH0 HASHK(H0)
 #define HASH1 HASHK(H1)
 #define HASH2 HASHK(H2)
 #define HASH3 HASHK(H3)
@@ -1087,6 +1131,7 @@ constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 
 static void ensure_attrs() {
     static int done_dev = -1;
     if (done_dev == ctx().device) return;
+    CUDA_CHECK(cudaFuncSetAttribute(HASH0, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H0_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(HASH1, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H1_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(HASH2, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H2_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(HASH3, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H3_SMEM)));
@@ -1161,20 +1206,20 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     LAUNCH_HASH(HASH3, H3, BIN_H3, 3)
     LAUNCH_HASH(HASH2, H2, BIN_H2, 4)
     LAUNCH_HASH(HASH1, H1, BIN_H1, 5)
+    LAUNCH_HASH(HASH0, H0, BIN_H0, 8)
 #undef LAUNCH_HASH
     // rows whose hash probes ran long: bitmap path
     DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 6);
-    count_launch(8);
+    count_launch(9);
     check_launch("block bins");
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
     t = ktime_begin("warp_bins", st);
-    warp_bin_kernel<16><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W16, scratch.p, soff.p, counts.p);
     warp_bin_kernel<8><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W8, scratch.p, soff.p, counts.p);
     warp_bin_kernel<4><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W4, scratch.p, soff.p, counts.p);
     warp_bin_kernel<2><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W2, scratch.p, soff.p, counts.p);
     warp_bin_kernel<1><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W1, scratch.p, soff.p, counts.p);
     ktime_end(t);
-    count_launch(5);
+    count_launch(4);
     check_launch("warp_bin_kernel");
     trace_mark("bin kernels");
     // 5. row offsets
@@ -1228,7 +1273,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
 
 void engine_thresholds(uint64_t* out, uint32_t* n) {
     // ub upper limits of bins W1, W2, W4, W8, W16, H1..H6 (DENSE above)
-    const uint64_t t[11] = {32, 64, 128, 256, kWarpMaxUb, kH1, kH2, kH3, kH4, kH5, kH6};
+    const uint64_t t[11] = {32, 64, 128, kWarpMaxUb, kH0, kH1, kH2, kH3, kH4, kH5, kH6};
     const uint32_t k = *n < 11 ? *n : 11;
     for (uint32_t i = 0; i < k; ++i) out[i] = t[i];
     *n = 11;
