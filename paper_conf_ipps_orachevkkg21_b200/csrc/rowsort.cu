@@ -360,6 +360,12 @@ __device__ __forceinline__ uint32_t vadd2(uint32_t a, uint32_t b) {  // per-16-b
     asm("add.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
     return r;
 }
+// *p = v if q (predicated store: no branch / reconvergence around it)
+__device__ __forceinline__ void st_if(idx_t* p, uint32_t v, bool q) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+                 "r"(uint32_t(q))
+                 : "memory");
+}
 constexpr uint32_t kOvfFlag = 0x80000000u;
 constexpr uint32_t kSlots = 16;
 
@@ -632,36 +638,47 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             // compacted, so slot s of bucket 2m goes to out[poff[m] + s] and of
             // bucket 2m+1 to out[poff[m] + count(2m) + s].  Each store writes two
             // runs of <= 16 consecutive columns.  The lane also restores its word.
-            const uint32_t sl = lane & 15u;
+            // lane = (pair g4 of 4, slots 2t and 2t+1): 8 lanes per pair, each
+            // reading two table words (banks 4t + g4 and 4t + g4 + 2: conflict-free
+            // with MPP = 2 mod 32) and storing up to 4 values
+            const uint32_t t8 = lane & 7u, g4 = lane >> 3;
 #pragma unroll 1
             for (uint32_t i = 0; i < KP; ++i) {
                 const uint32_t mb = i * THREADS + wib * 32;
+                if (mb >= np) break;
+                const uint32_t jn = min(32u, np - mb);
 #pragma unroll 1
-                for (uint32_t j = 0; j < 32 && mb + j < np; j += 2) {
-                    const uint32_t m = mb + j + (lane >> 4);
-                    if (m < np) {
-                        const uint32_t w = tabw[sl * MPP + m];
-                        tabw[sl * MPP + m] = 0xFFFFFFFFu;
-                        const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
-                        const uint32_t c0 = bucket_count(nn.x);
-                        idx_t* o = out + poff[m];
-                        const idx_t base0 = clo + 2 * m * W;
-                        const uint32_t v0 = w & 0xFFFFu, v1 = w >> 16;
-                        if (v0 != 0xFFFFu) o[sl] = base0 + v0;
-                        if (v1 != 0xFFFFu) o[c0 + sl] = base0 + W + v1;
-                        if (sl == 0) {
-                            if ((nn.x | nn.y) & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
-                                if (nn.x & kOvfFlag) {
-                                    const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
-                                    for (uint32_t q = kSlots; q < mc; ++q) o[q] = base0 + pool[off + q - kSlots];
-                                }
-                                if (nn.y & kOvfFlag) {
-                                    const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
-                                    for (uint32_t q = kSlots; q < mc; ++q) o[c0 + q] = base0 + W + pool[off + q - kSlots];
-                                }
+                for (uint32_t j = 0; j < jn; j += 4) {
+                    // past the last pair a lane group repeats pair mb+j and stores
+                    // nothing (its restores write the same clean values)
+                    const bool ok = j + g4 < jn;
+                    const uint32_t m = mb + j + (ok ? g4 : 0u);
+                    uint32_t* wp = tabw + (2 * t8) * MPP + m;
+                    const uint32_t wa = wp[0], wb = wp[MPP];
+                    wp[0] = 0xFFFFFFFFu;
+                    wp[MPP] = 0xFFFFFFFFu;
+                    const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
+                    const uint32_t pm = poff[m];
+                    const uint32_t c0 = (nn.x & kOvfFlag) ? obcnt[nn.x & ~kOvfFlag] >> 16 : nn.x;
+                    const uint32_t base0 = clo + m * (2 * W), base1 = base0 + W;
+                    idx_t* o0 = out + (pm + 2 * t8);
+                    idx_t* o1 = out + (pm + c0 + 2 * t8);
+                    st_if(o0, base0 + (wa & 0xFFFFu), ok && (wa & 0xFFFFu) != 0xFFFFu);
+                    st_if(o0 + 1, base0 + (wb & 0xFFFFu), ok && (wb & 0xFFFFu) != 0xFFFFu);
+                    st_if(o1, base1 + (wa >> 16), ok && (wa >> 16) != 0xFFFFu);
+                    st_if(o1 + 1, base1 + (wb >> 16), ok && (wb >> 16) != 0xFFFFu);
+                    if (ok && t8 == 0) {
+                        if ((nn.x | nn.y) & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
+                            if (nn.x & kOvfFlag) {
+                                const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                                for (uint32_t q = kSlots; q < mc; ++q) out[pm + q] = base0 + pool[off + q - kSlots];
                             }
-                            reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
+                            if (nn.y & kOvfFlag) {
+                                const uint32_t e = obcnt[nn.y & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
+                                for (uint32_t q = kSlots; q < mc; ++q) out[pm + c0 + q] = base1 + pool[off + q - kSlots];
+                            }
                         }
+                        reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
                     }
                 }
             }
