@@ -638,35 +638,37 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             // compacted, so slot s of bucket 2m goes to out[poff[m] + s] and of
             // bucket 2m+1 to out[poff[m] + count(2m) + s].  Each store writes two
             // runs of <= 16 consecutive columns.  The lane also restores its word.
-            // lane = (pair g4 of 4, slots 2t and 2t+1): 8 lanes per pair, each
-            // reading two table words (banks 4t + g4 and 4t + g4 + 2: conflict-free
-            // with MPP = 2 mod 32) and storing up to 4 values
-            const uint32_t t8 = lane & 7u, g4 = lane >> 3;
+            // lane = (pair g of 8, slots 4t .. 4t+3): 4 lanes per pair, each
+            // reading four table words (banks 8t + 2k + g: conflict-free with
+            // MPP = 2 mod 32) and storing up to 8 values
+            const uint32_t t8 = lane & 3u, g4 = lane >> 2;
 #pragma unroll 1
             for (uint32_t i = 0; i < KP; ++i) {
                 const uint32_t mb = i * THREADS + wib * 32;
                 if (mb >= np) break;
                 const uint32_t jn = min(32u, np - mb);
 #pragma unroll 1
-                for (uint32_t j = 0; j < jn; j += 4) {
+                for (uint32_t j = 0; j < jn; j += 8) {
                     // past the last pair a lane group repeats pair mb+j and stores
                     // nothing (its restores write the same clean values)
                     const bool ok = j + g4 < jn;
                     const uint32_t m = mb + j + (ok ? g4 : 0u);
-                    uint32_t* wp = tabw + (2 * t8) * MPP + m;
-                    const uint32_t wa = wp[0], wb = wp[MPP];
-                    wp[0] = 0xFFFFFFFFu;
-                    wp[MPP] = 0xFFFFFFFFu;
+                    uint32_t* wp = tabw + (4 * t8) * MPP + m;
+                    uint32_t wv[4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) wv[k] = wp[k * MPP];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) wp[k * MPP] = 0xFFFFFFFFu;
                     const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
                     const uint32_t pm = poff[m];
                     const uint32_t c0 = (nn.x & kOvfFlag) ? obcnt[nn.x & ~kOvfFlag] >> 16 : nn.x;
                     const uint32_t base0 = clo + m * (2 * W), base1 = base0 + W;
-                    idx_t* o0 = out + (pm + 2 * t8);
-                    idx_t* o1 = out + (pm + c0 + 2 * t8);
-                    st_if(o0, base0 + (wa & 0xFFFFu), ok && (wa & 0xFFFFu) != 0xFFFFu);
-                    st_if(o0 + 1, base0 + (wb & 0xFFFFu), ok && (wb & 0xFFFFu) != 0xFFFFu);
-                    st_if(o1, base1 + (wa >> 16), ok && (wa >> 16) != 0xFFFFu);
-                    st_if(o1 + 1, base1 + (wb >> 16), ok && (wb >> 16) != 0xFFFFu);
+                    idx_t* o0 = out + (pm + 4 * t8);
+                    idx_t* o1 = out + (pm + c0 + 4 * t8);
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) st_if(o0 + k, base0 + (wv[k] & 0xFFFFu), ok && (wv[k] & 0xFFFFu) != 0xFFFFu);
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) st_if(o1 + k, base1 + (wv[k] >> 16), ok && (wv[k] >> 16) != 0xFFFFu);
                     if (ok && t8 == 0) {
                         if ((nn.x | nn.y) & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
                             if (nn.x & kOvfFlag) {
