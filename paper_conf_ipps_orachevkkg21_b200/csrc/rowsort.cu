@@ -1022,11 +1022,15 @@ __global__ void tile_deps_kernel(const uint64_t* __restrict__ src_lo, uint64_t n
     }
 }
 
-__global__ void __launch_bounds__(kCThreads)
+__global__ void __launch_bounds__(kCThreads, 4)
 compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint64_t* __restrict__ rowptr,
                        const uint32_t* __restrict__ tile_row, const uint2* __restrict__ wait_range,
                        idx_t nrows, uint64_t nnz, uint32_t* flags, uint32_t* ticket) {
-    __shared__ uint64_t s_rp[kCStage + 1], s_sl[kCStage];
+    // staged rows of the tile in tile-local coordinates: s_beg[i] = start of
+    // row r0+i relative to d0 (clamped to 0), s_beg[nr] = kCT; s_src[i] =
+    // source pointer of tile-local position 0 for that row (buf + d0 + slack)
+    __shared__ int32_t s_beg[kCStage + 1];
+    __shared__ const idx_t* s_src[kCStage];
     __shared__ uint32_t s_t, s_r0, s_r1;
     __shared__ uint2 s_w;
     const uint64_t ntiles = (nnz + kCT - 1) / kCT;
@@ -1044,7 +1048,8 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
         __syncthreads();
         const uint32_t t = s_t;
         if (t >= ntiles) break;
-        const uint64_t d0 = uint64_t(t) * kCT, d1 = min(d0 + kCT, nnz);
+        const uint64_t d0 = uint64_t(t) * kCT;
+        const uint32_t n = uint32_t(min(uint64_t(kCT), nnz - d0));  // tile length
         const uint32_t r0 = s_r0, r1 = s_r1;
         const uint64_t slack1 = soff[r1] - rowptr[r1];
         if (slack1 == 0) {  // whole tile already in place (slack is nondecreasing)
@@ -1057,33 +1062,44 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
         if (staged) {
             for (uint32_t i = threadIdx.x; i < nr; i += kCThreads) {
                 const uint64_t rp = rowptr[r0 + i];
-                s_rp[i] = rp;
-                s_sl[i] = soff[r0 + i] - rp;
+                s_beg[i] = rp <= d0 ? 0 : int32_t(min(rp - d0, uint64_t(kCT)));
+                s_src[i] = buf + (d0 + (soff[r0 + i] - rp));
             }
+            if (threadIdx.x == 0) s_beg[nr] = int32_t(kCT);
         }
         __syncthreads();
         idx_t v[kCItems];
-        uint32_t ri = 0;  // staged: row index relative to r0, advanced monotonically
+        if (staged) {
+            // element e = k*kCThreads + t of the tile; the row advances rarely
+            // (rows average thousands of elements), by binary search over the
+            // staged starts when it does
+            uint32_t ri = 0;
+            int32_t nxt = s_beg[1];
+            const idx_t* sp = s_src[0];
 #pragma unroll
-        for (int k = 0; k < kCItems; ++k) {
-            const uint64_t d = d0 + uint32_t(k) * kCThreads + threadIdx.x;
-            if (d < d1) {
-                uint64_t src;
-                if (staged) {
-                    if (ri + 1 < nr && s_rp[ri + 1] <= d) {  // next row(s): binary search in smem
-                        uint32_t lo = ri + 1, hi = nr - 1;
-                        while (lo < hi) {
-                            const uint32_t mid = (lo + hi + 1) >> 1;
-                            if (s_rp[mid] <= d) lo = mid; else hi = mid - 1;
-                        }
-                        ri = lo;
+            for (int k = 0; k < kCItems; ++k) {
+                const int32_t e = k * kCThreads + int32_t(threadIdx.x);
+                if (e >= nxt) {
+                    uint32_t lo = ri + 1, hi = nr - 1;  // last row with start <= e
+                    while (lo < hi) {
+                        const uint32_t mid = (lo + hi + 1) >> 1;
+                        if (s_beg[mid] <= e) lo = mid; else hi = mid - 1;
                     }
-                    src = d + s_sl[ri];
-                } else {
-                    const uint32_t r = row_of(rowptr, r0, r1, d);
-                    src = d + (soff[r] - rowptr[r]);
+                    ri = lo;
+                    nxt = s_beg[ri + 1];
+                    sp = s_src[ri];
                 }
-                v[k] = buf[src];
+                if (uint32_t(e) < n) v[k] = sp[e];
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < kCItems; ++k) {
+                const uint32_t e = k * kCThreads + threadIdx.x;
+                if (e < n) {
+                    const uint64_t d = d0 + e;
+                    const uint32_t r = row_of(rowptr, r0, r1, d);
+                    v[k] = buf[d + (soff[r] - rowptr[r])];
+                }
             }
         }
         // publish "read done": the barrier orders every thread's loads before
@@ -1097,12 +1113,11 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
         for (uint32_t j = s_w.x + threadIdx.x; j < s_w.y; j += kCThreads)
             while (ld_acquire_u32(&flags[j]) == 0) __nanosleep(64);
         __syncthreads();
+        idx_t* dp = buf + d0 + threadIdx.x;
 #pragma unroll
-        for (int k = 0; k < kCItems; ++k) {
-            const uint64_t d = d0 + uint32_t(k) * kCThreads + threadIdx.x;
-            if (d < d1) buf[d] = v[k];
-        }
-        __syncthreads();  // s_rp / s_t reuse
+        for (int k = 0; k < kCItems; ++k)
+            if (k * kCThreads + threadIdx.x < n) dp[k * kCThreads] = v[k];
+        __syncthreads();  // s_beg / s_t reuse
     }
 }
 
