@@ -383,7 +383,7 @@ __host__ __device__ constexpr uint32_t first_entries(uint64_t maxub) { return ui
 //               ovl[OVCAP] | pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | poff[MAXB/2]
 // (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
 // which are dead once the products are inserted: BATCH * 3 >= THREADS)
-template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU>
+template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU, bool DEDUP_B>
 __global__ void __launch_bounds__(THREADS, MINB)
 hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
                 const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
@@ -499,10 +499,12 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         bool fallback = s_flag != 0;  // overflow list full: the row goes to the bitmap bin
         if (!fallback) {
             // ---- pass A: sort each owned bucket pair in 16x2 SIMD ----------------
-            // Duplicates are removed in registers (rare: replaced by 0xFFFF and
-            // re-sorted), so every bucket leaves pass A as its distinct values
-            // in slots [0, count) followed by 0xFFFF; bcnt[b] becomes the
-            // bucket's distinct count, or kOvfFlag | list index
+            // Every bucket leaves pass A sorted (duplicates adjacent, empty
+            // 0xFFFF slots last; DEDUP_B = false: duplicates already replaced by
+            // 0xFFFF and re-sorted here, the better choice for the small
+            // bins); bcnt[b] becomes the bucket's distinct count,
+            // or kOvfFlag | list index (the overflow pass then leaves the first
+            // 16 distinct values in its slots)
 #pragma unroll 1
             for (uint32_t m = threadIdx.x; m < np; m += THREADS) {
                 const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
@@ -530,7 +532,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                 uint32_t dsum = 0;
 #pragma unroll
                 for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
-                if (dsum) {  // drop the duplicates: mark them empty, sort again
+                if (!DEDUP_B && dsum) {  // drop the duplicates here: mark them empty, sort again
                     uint32_t prev = x[0];
 #pragma unroll
                     for (int k2 = 1; k2 < 16; ++k2) {
@@ -640,7 +642,12 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             // runs of <= 16 consecutive columns.  The lane also restores its word.
             // lane = (pair g of 8, slots 4t .. 4t+3): 4 lanes per pair, each
             // reading four table words (banks 8t + 2k + g: conflict-free with
-            // MPP = 2 mod 32) and storing up to 8 values
+            // MPP = 2 mod 32) and storing up to 8 values.  A word holds slot s
+            // of both buckets of the pair, so the dedup runs in 16x2 SIMD: a
+            // slot is kept if valid and not equal to the previous slot (the
+            // previous lane's last word for k = 0); its output position is the
+            // number of kept slots before it (packed per-bucket counts,
+            // exclusive scan over the pair's 4 lanes)
             const uint32_t t8 = lane & 3u, g4 = lane >> 2;
 #pragma unroll 1
             for (uint32_t i = 0; i < KP; ++i) {
@@ -659,16 +666,43 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                     for (int k = 0; k < 4; ++k) wv[k] = wp[k * MPP];
 #pragma unroll
                     for (int k = 0; k < 4; ++k) wp[k * MPP] = 0xFFFFFFFFu;
+                    uint32_t inc[4], ex;
+                    if (DEDUP_B) {
+                        uint32_t prevw = __shfl_up_sync(FULL, wv[3], 1, 4);
+                        if (t8 == 0) prevw = 0xFFFFFFFFu;
+                        uint32_t keep[4], cnt = 0;
+#pragma unroll
+                        for (int k = 0; k < 4; ++k)
+                            keep[k] = __vcmpne2(wv[k], 0xFFFFFFFFu) & ~__vcmpeq2(wv[k], k ? wv[k - 1] : prevw);
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            inc[k] = cnt;  // kept slots of this lane before slot k (packed)
+                            cnt += keep[k] & 0x00010001u;
+                            wv[k] |= ~keep[k];  // dropped slots read as empty below
+                        }
+                        uint32_t sc = cnt;  // inclusive scan of the packed counts over the 4 lanes
+                        uint32_t y = __shfl_up_sync(FULL, sc, 1, 4);
+                        if (t8 >= 1) sc += y;
+                        y = __shfl_up_sync(FULL, sc, 2, 4);
+                        if (t8 >= 2) sc += y;
+                        ex = sc - cnt;
+                    } else {  // buckets already compacted: slot s goes to position s
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) inc[k] = uint32_t(k) * 0x00010001u;
+                        ex = 4 * t8 * 0x00010001u;
+                    }
                     const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
                     const uint32_t pm = poff[m];
                     const uint32_t c0 = (nn.x & kOvfFlag) ? obcnt[nn.x & ~kOvfFlag] >> 16 : nn.x;
                     const uint32_t base0 = clo + m * (2 * W), base1 = base0 + W;
-                    idx_t* o0 = out + (pm + 4 * t8);
-                    idx_t* o1 = out + (pm + c0 + 4 * t8);
+                    idx_t* o0 = out + (pm + (ex & 0xFFFFu));
+                    idx_t* o1 = out + (pm + c0 + (ex >> 16));
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) st_if(o0 + k, base0 + (wv[k] & 0xFFFFu), ok && (wv[k] & 0xFFFFu) != 0xFFFFu);
+                    for (int k = 0; k < 4; ++k)
+                        st_if(o0 + (inc[k] & 0xFFFFu), base0 + (wv[k] & 0xFFFFu), ok && (wv[k] & 0xFFFFu) != 0xFFFFu);
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) st_if(o1 + k, base1 + (wv[k] >> 16), ok && (wv[k] >> 16) != 0xFFFFu);
+                    for (int k = 0; k < 4; ++k)
+                        st_if(o1 + (inc[k] >> 16), base1 + (wv[k] >> 16), ok && (wv[k] >> 16) != 0xFFFFu);
                     if (ok && t8 == 0) {
                         if ((nn.x | nn.y) & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
                             if (nn.x & kOvfFlag) {
@@ -1135,23 +1169,25 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
            batch * kSegBytes + first_entries(uint64_t(buckets) * 8) * sizeof(uint32_t) +
            ovcap * (sizeof(idx_t) + sizeof(uint16_t)) + obcap * 2 * sizeof(uint32_t);
 }
-#define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U)                                           \
+#define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U, DB)                                       \
     constexpr int NAME##_T = T, NAME##_PERSM = PERSM, NAME##_U = U;                                \
+    constexpr bool NAME##_DB = DB;                                                                 \
     constexpr uint32_t NAME##_B = uint32_t(UB / 8), NAME##_OVCAP = OVCAP, NAME##_OBCAP = OBCAP,     \
                        NAME##_BATCH = BATCH;                                                       \
     constexpr size_t NAME##_SMEM = hash_smem(T, BATCH, uint32_t(UB / 8), OVCAP, OBCAP);            \
     static_assert(PERSM * (NAME##_SMEM + 1024 + 1200) <= 228 * 1024, #NAME " residency");         \
     static_assert(PERSM * T <= 2048, #NAME " threads");
-// <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread>
+// <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread,
+//  dedup in pass B (else re-sort in pass A)>
 // (expected per row at mean load 8 with 16 slots: list ~ub/1500, buckets ~ub/2000)
-HBIN(H0, 32, kH0, 32, 16, 64, 32, 4)
-HBIN(H1, 64, kH1, 32, 16, 128, 20, 4)
-HBIN(H2, 64, kH2, 32, 16, 128, 16, 4)
-HBIN(H3, 128, kH3, 64, 32, 256, 8, 4)
-HBIN(H4, 256, kH4, 64, 32, 256, 4, 8)
-HBIN(H5, 512, kH5, 128, 64, 256, 2, 8)
-HBIN(H6, 1024, kH6, 192, 96, 384, 1, 8)
-#define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U>
+HBIN(H0, 32, kH0, 32, 16, 64, 32, 4, false)
+HBIN(H1, 64, kH1, 32, 16, 128, 20, 4, false)
+HBIN(H2, 64, kH2, 32, 16, 128, 16, 4, false)
+HBIN(H3, 128, kH3, 64, 32, 256, 8, 4, false)
+HBIN(H4, 256, kH4, 64, 32, 256, 4, 8, true)
+HBIN(H5, 512, kH5, 128, 64, 256, 2, 8, true)
+HBIN(H6, 1024, kH6, 192, 96, 384, 1, 8, true)
+#define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U, N##_DB>
 #define HASH0 HASHK(H0)
 #define HASH1 HASHK(H1)
 #define HASH2 HASHK(H2)
