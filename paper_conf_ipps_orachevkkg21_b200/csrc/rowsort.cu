@@ -152,9 +152,27 @@ __device__ __forceinline__ uint32_t warp_flat(const idx_t* p, uint32_t len, F&& 
 // non-empty segment); replaces the binary search of the gather.
 // Returns the number of products in the batch; ends with a barrier.
 constexpr uint32_t kFirstShift = 6;
+// descriptor-mode segment base of row r: its descriptors are desc[seg_base + j]
+__device__ __forceinline__ uint64_t seg_base(const SegSource& s, idx_t r) {
+    return s.kind == 1 ? 0 : s.dbase[r] + r;
+}
+// stage one descriptor as entry i of the batch whose concatenation starts at base
+__device__ __forceinline__ void stage_one(const uint4& e, uint32_t i, uint32_t base, const idx_t** sd_ptr,
+                                          uint32_t* sd_end, uint32_t* sd_first) {
+    const idx_t* p = reinterpret_cast<const idx_t*>((uint64_t(e.y) << 32) | e.x);
+    const uint32_t end = e.w - base, start = end - e.z;
+    sd_ptr[i] = p - start;
+    sd_end[i] = end;
+    if (sd_first) {
+#pragma unroll 1
+        for (uint32_t j = (start + (1u << kFirstShift) - 1) >> kFirstShift; (j << kFirstShift) < end; ++j)
+            sd_first[j] = i;
+    }
+}
 template <int THREADS>
-__device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint32_t s0, uint32_t n,
-                                                   const idx_t** sd_ptr, uint32_t* sd_end, uint32_t* sd_first) {
+__device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint64_t sbase, uint32_t s0,
+                                                   uint32_t n, const idx_t** sd_ptr, uint32_t* sd_end,
+                                                   uint32_t* sd_first) {
     if (s.kind == 1) {  // one segment
         if (threadIdx.x == 0) {
             const off_t64 b = s.lrp[r];
@@ -164,21 +182,10 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
         __syncthreads();
         return sd_end[0];
     }
-    const uint4* d = s.desc + (s.dbase[r] + r + s0);
-    const uint32_t base = s0 ? s.desc[s.dbase[r] + r + s0 - 1].w : 0u;
+    const uint4* d = s.desc + (sbase + s0);
+    const uint32_t base = s0 ? s.desc[sbase + s0 - 1].w : 0u;
 #pragma unroll 1
-    for (uint32_t i = threadIdx.x; i < n; i += THREADS) {
-        const uint4 e = d[i];
-        const idx_t* p = reinterpret_cast<const idx_t*>((uint64_t(e.y) << 32) | e.x);
-        const uint32_t end = e.w - base, start = end - e.z;
-        sd_ptr[i] = p - start;
-        sd_end[i] = end;
-        if (sd_first) {
-#pragma unroll 1
-            for (uint32_t j = (start + (1u << kFirstShift) - 1) >> kFirstShift; (j << kFirstShift) < end; ++j)
-                sd_first[j] = i;
-        }
-    }
+    for (uint32_t i = threadIdx.x; i < n; i += THREADS) stage_one(d[i], i, base, sd_ptr, sd_end, sd_first);
     __syncthreads();
     return d[n - 1].w - base;
 }
@@ -191,13 +198,16 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
 // crosses more than one boundary); the U loads are issued before any
 // insert.  A warp covers 32*U consecutive products, i.e. a few sectors of
 // each B row.  Ends with a barrier.
+// prestaged: the first batch is already staged (and visible to all threads).
 template <int THREADS, int U, typename F>
-__device__ __forceinline__ void block_products(const SegSource& s, idx_t r, const idx_t** sd_ptr,
-                                               uint32_t* sd_end, uint32_t* sd_first, uint32_t batch, F&& f) {
-    const uint32_t nseg = num_segs(s, r);
+__device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint64_t sbase, uint32_t nseg,
+                                               const idx_t** sd_ptr, uint32_t* sd_end, uint32_t* sd_first,
+                                               uint32_t batch, bool prestaged, F&& f) {
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
         const uint32_t ns = min(batch, nseg - s0);
-        const uint32_t total = stage_segments<THREADS>(s, r, s0, ns, sd_ptr, sd_end, sd_first);
+        const uint32_t total = (s0 == 0 && prestaged)
+                                   ? sd_end[ns - 1]
+                                   : stage_segments<THREADS>(s, r, sbase, s0, ns, sd_ptr, sd_end, sd_first);
 #ifdef SPBLA_PROBE
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
@@ -372,22 +382,73 @@ constexpr uint32_t kSlots = 16;
 template <int E>
 __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]);
 
+// Per-row work record of the hash bins (written by make_recs_kernel after
+// binning): one 40-B load gives everything the row needs.
+struct RowRec {
+    uint32_t r, u, clo, chi;  // row, upper bound, column span [clo, chi]
+    uint64_t out, seg;        // scratch offset, descriptor base (kind 0)
+    uint32_t nseg, pad;
+};
+// A row's plan, computed once by thread 0 (one row ahead) and read by all
+// threads from shared memory: mode, bucket count, width and exact reciprocal.
+enum : uint32_t { kPlanHash = 0, kPlanBitmap = 1, kPlanWide = 2, kPlanEnd = 3 };
+struct RowPlan {
+    RowRec rec;
+    uint32_t mode, nb, W, l, M, nw;
+};
+template <uint32_t MAXB>
+__device__ __forceinline__ RowPlan make_plan(const RowRec& x) {
+    RowPlan P;
+    P.rec = x;
+    const uint64_t span = uint64_t(x.chi) - x.clo + 1;
+    // nb buckets of width W <= 65535 (16-bit offsets); too wide a span for the
+    // table goes to the bitmap bin.  nb is even (buckets are sorted in pairs).
+    const uint64_t nbw = (span + 65534) / 65535;
+    const uint32_t nb =
+        (uint32_t(min(max(max(uint64_t((x.u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB))) + 1) & ~1u;
+    const uint64_t words = (span + 31) >> 5;
+    P.nb = nb;
+    P.nw = uint32_t(min(words, uint64_t(0xFFFFFFFFu)));
+    P.W = P.l = P.M = 0;
+    if (words <= 9ull * nb) {  // the span bitmap is no larger than the table
+        P.mode = kPlanBitmap;
+    } else if (nbw > MAXB) {  // span too wide for 16-bit offsets in this table
+        P.mode = kPlanWide;
+    } else {
+        // bucket width W (> 288 here: smaller spans took the bitmap) and an exact
+        // 32-bit reciprocal: d < nb*W < 2^29, M = ceil(2^(32+l) / W) with
+        // 2^(l+3) >= W gives floor(d / W) = umulhi(d, M) >> l (M < 2^30)
+        P.mode = kPlanHash;
+        P.W = uint32_t((span + nb - 1) / nb);
+        P.l = (32 - __clz(P.W - 1)) - 3;
+        P.M = uint32_t(((uint64_t(1) << (32 + P.l)) + P.W - 1) / P.W);
+    }
+    return P;
+}
+
 // Pair stride of the slot-major table: MPP = 2 (mod 32), so slot s of pair m
 // sits in bank 2s + m (mod 32): the per-thread pass A (lanes = consecutive
-// pairs, one slot) and the warp-cooperative pass B (lanes = 16 slots x 2
+// pairs, one slot) and the warp-cooperative pass B (lanes = 4 slots x 8
 // consecutive pairs) are both conflict-free.
 __host__ __device__ constexpr uint32_t pair_stride(uint32_t mp) { return ((mp + 29) / 32) * 32 + 2; }
 __host__ __device__ constexpr uint32_t first_entries(uint64_t maxub) { return uint32_t((maxub >> kFirstShift) + 1); }
 
+// Rows flow through a 3-stage software pipeline (one block, rows claimed
+// from an atomic counter): while row i runs, thread 0 holds the claim of row
+// i+2, loads row i+1's record at row start and publishes its plan after the
+// gather; after pass A every thread issues the loads of row i+1's first
+// descriptor batch and stages it at the end of row i.  A row therefore starts
+// with its metadata and descriptors already in shared memory: no global
+// round trip and no staging barrier before its gather.
+//
 // dynamic smem: tabw[16*MPP] | bcnt[MAXB] | sd_ptr[BATCH] | sd_end[BATCH] | sd_first[NF] |
 //               ovl[OVCAP] | pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | poff[MAXB/2]
 // (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
 // which are dead once the products are inserted: BATCH * 3 >= THREADS)
 template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU, bool DEDUP_B>
 __global__ void __launch_bounds__(THREADS, MINB)
-hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
-                const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
-                idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts,
+hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* __restrict__ bounds,
+                idx_t* __restrict__ scratch, uint32_t* __restrict__ counts,
                 uint32_t* __restrict__ work, idx_t* __restrict__ ovf_rows, uint32_t* __restrict__ ovf_cnt) {
     constexpr int NW = THREADS / 32;
     constexpr uint32_t MP = MAXB / 2;                      // bucket pairs
@@ -395,6 +456,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     constexpr uint32_t TABW = 16 * MPP;                    // table words
     constexpr uint32_t KP = (MP + THREADS - 1) / THREADS;  // pairs per thread
     constexpr uint32_t NF = first_entries(uint64_t(MAXB) * 8);
+    constexpr int PF = (BATCH + THREADS - 1) / THREADS;    // prefetched descriptors per thread
     extern __shared__ __align__(16) unsigned char smem_raw[];
     uint32_t* tabw = reinterpret_cast<uint32_t*>(smem_raw);  // word s*MPP + m = slot s of pair m
     uint16_t* tab16 = reinterpret_cast<uint16_t*>(smem_raw);
@@ -412,79 +474,123 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
     static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0 && MP % 32 == 0, "hash bin layout");
     __shared__ uint32_t s_w[33];
     __shared__ uint32_t s_wt[KP][NW];
-    __shared__ uint32_t s_item[2], s_flag, s_novf, s_nob, s_pool;
+    __shared__ uint32_t s_flag, s_novf, s_nob, s_pool;
+    __shared__ RowPlan s_plan[2];
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
+    const bool pre = src.kind == 0;  // descriptor mode: first batches are prefetched
+    RowPlan end_plan;
+    end_plan.mode = kPlanEnd;
+    // descriptor prefetch of a row's first batch: issue (loads in flight) ...
+    uint4 pfd[PF];
+    auto pf_issue = [&](const RowPlan& N) {
+        if (!pre || N.mode == kPlanEnd) return;
+        const uint32_t n = min(N.rec.nseg, BATCH);
+#pragma unroll
+        for (int k = 0; k < PF; ++k) {
+            const uint32_t i = threadIdx.x + k * THREADS;
+            if (i < n) pfd[k] = src.desc[N.rec.seg + i];
+        }
+    };
+    // ... and commit (staged into the descriptor arrays; visible after the next barrier)
+    auto pf_commit = [&](const RowPlan& N) {
+        if (!pre || N.mode == kPlanEnd) return;
+        const uint32_t n = min(N.rec.nseg, BATCH);
+#pragma unroll
+        for (int k = 0; k < PF; ++k) {
+            const uint32_t i = threadIdx.x + k * THREADS;
+            if (i < n) stage_one(pfd[k], i, 0u, sd_ptr, sd_end, sd_first);
+        }
+    };
     // the table is kept clean between rows (all slots 0xFFFF, counters 0):
     // every row restores what it dirtied before the end-of-row barrier
 #pragma unroll 1
     for (uint32_t i = threadIdx.x; i < TABW; i += THREADS) tabw[i] = 0xFFFFFFFFu;
 #pragma unroll 1
     for (uint32_t i = threadIdx.x; i < MAXB; i += THREADS) bcnt[i] = 0u;
-    if (threadIdx.x == 0) s_item[0] = lo_i + atomicAdd(work, 1u);
+    // prologue: claim rows 0 and 1, plan row 0, stage its first batch
+    // the pipeline thread is the last one: it has the least pass-A work
+    constexpr unsigned PT = THREADS - 1;
+    uint32_t nxt1 = 0, nxt2 = 0;  // (thread PT) claimed items of rows i+1 and i+2
+    if (threadIdx.x == PT) {
+        const uint32_t i0 = lo_i + atomicAdd(work, 1u);
+        nxt1 = lo_i + atomicAdd(work, 1u);
+        s_plan[0] = i0 < hi_i ? make_plan<MAXB>(recs[i0]) : end_plan;
+    }
+    __syncthreads();
+    {
+        const RowPlan P0 = s_plan[0];
+        pf_issue(P0);
+        pf_commit(P0);
+    }
     __syncthreads();
     PROBE_DECL
 #pragma unroll 1
     for (uint32_t it = 0;; ++it) {
-        // the next row is claimed while this one runs: one barrier per row boundary
-        const uint32_t item = s_item[it & 1];
-        if (item >= hi_i) break;
+        const RowPlan P = s_plan[it & 1];
+        if (P.mode == kPlanEnd) break;
+        RowRec nx;
+        bool have_nx = false;
+        if (threadIdx.x == PT) {
+            nxt2 = lo_i + atomicAdd(work, 1u);
+            have_nx = nxt1 < hi_i;
+            if (have_nx) nx = recs[nxt1];
+        }
         if (threadIdx.x == 0) {
-            s_item[(it + 1) & 1] = lo_i + atomicAdd(work, 1u);
             s_flag = 0;
             s_novf = 0;
             s_nob = 0;
             s_pool = 0;
         }
+        // thread PT: plan of row i+1 into s_plan (visible after the next barrier)
+        auto publish_next = [&]() {
+            if (threadIdx.x == PT) {
+                s_plan[(it + 1) & 1] = have_nx ? make_plan<MAXB>(nx) : end_plan;
+                nxt1 = nxt2;
+            }
+        };
         PROBE(0);
-        const idx_t r = rows[item];
-        const uint32_t u = uint32_t(ub[r]);
-        uint32_t clo = 0, chi = ncols - 1;
-        if (range) {
-            const uint2 rg = range[r];
-            clo = rg.x;
-            chi = rg.y;
-        }
-        const uint64_t span = uint64_t(chi) - clo + 1;
-        // nb buckets of width W <= 65535 (16-bit offsets); too wide a span for the
-        // table goes to the bitmap bin.  nb is even (buckets are sorted in pairs).
-        const uint64_t nbw = (span + 65534) / 65535;
-        const uint32_t nb =
-            (uint32_t(min(max(max(uint64_t((u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB))) + 1) & ~1u;
-        const uint32_t np = nb / 2;
-        const uint64_t words = (span + 31) >> 5;
-        idx_t* out = scratch + soff[r];
-        if (words <= 9ull * nb) {  // the span bitmap is no larger than the table
-            const uint32_t nw = uint32_t(words);
+        const idx_t r = P.rec.r;
+        const uint32_t clo = P.rec.clo;
+        const uint32_t nb = P.nb, np = nb / 2;
+        idx_t* out = scratch + P.rec.out;
+        if (P.mode == kPlanBitmap) {
+            const uint32_t nw = P.nw;
 #pragma unroll 1
             for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = 0u;
             __syncthreads();
-            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, sd_first, BATCH, [&](idx_t c) {
-                const uint32_t d = c - clo;
-                atomicOr(&bmw[d >> 5], 1u << (d & 31));
-            });
-            const uint32_t n = emit_bitmap<NW>(bmw, nw, clo, out, s_w);
+            block_products<THREADS, FLATU>(src, r, P.rec.seg, P.rec.nseg, sd_ptr, sd_end, sd_first, BATCH, pre,
+                                           [&](idx_t c) {
+                                               const uint32_t d = c - clo;
+                                               atomicOr(&bmw[d >> 5], 1u << (d & 31));
+                                           });
+            publish_next();
+            const uint32_t n = emit_bitmap<NW>(bmw, nw, clo, out, s_w);  // (barriers inside)
             if (threadIdx.x == 0) counts[r] = n;
 #pragma unroll 1
             for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = i < TABW ? 0xFFFFFFFFu : 0u;
+            const RowPlan N = s_plan[(it + 1) & 1];
+            pf_issue(N);
+            pf_commit(N);
             __syncthreads();
             continue;
         }
         PROBE(1);
-        if (nbw > MAXB) {  // span too wide for 16-bit offsets in this table
+        if (P.mode == kPlanWide) {
             if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            publish_next();
+            __syncthreads();
+            const RowPlan N = s_plan[(it + 1) & 1];
+            pf_issue(N);
+            pf_commit(N);
             __syncthreads();
             continue;
         }
-        // bucket width W (> 288 here: smaller spans took the bitmap) and an exact
-        // 32-bit reciprocal: d < nb*W < 2^29, M = ceil(2^(32+l) / W) with
-        // 2^(l+3) >= W gives floor(d / W) = umulhi(d, M) >> l (M < 2^30)
-        const uint32_t W = uint32_t((span + nb - 1) / nb);
-        const uint32_t l = (32 - __clz(W - 1)) - 3;
-        const uint32_t M = uint32_t(((uint64_t(1) << (32 + l)) + W - 1) / W);
+        const uint32_t W = P.W, l = P.l, M = P.M;
         PROBE(2);
-        block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, sd_first, BATCH, [&](idx_t c) {
+        block_products<THREADS, FLATU>(src, r, P.rec.seg, P.rec.nseg, sd_ptr, sd_end, sd_first, BATCH, pre,
+                                       [&](idx_t c) {
             const uint32_t d = c - clo;
             const uint32_t b = __umulhi(d, M) >> l;
             const uint32_t slot = atomicAdd(&bcnt[b], 1u);
@@ -550,9 +656,15 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
 #pragma unroll
                 for (int sl = 0; sl < 16; ++sl) tabw[sl * MPP + m] = (x[sl] & keep) | (tabw[sl * MPP + m] & ~keep);
             }
+            publish_next();  // (after PT's pass-A share, which is the smallest)
             __syncthreads();
             fallback = s_flag != 0;
+        } else {
+            publish_next();
+            __syncthreads();  // (the published plan of row i+1 becomes visible)
         }
+        const RowPlan N = s_plan[(it + 1) & 1];
+        pf_issue(N);  // row i+1's first descriptor batch: loads in flight through the rest of the row
         const uint32_t nob = s_nob;
         if (!fallback && nob) {
             // ---- overflow buckets: one warp each, <= 32 values sorted across lanes
@@ -718,9 +830,10 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
                     }
                 }
             }
+            pf_commit(N);
             __syncthreads();
             PROBE(7);
-            PROBE_PRINT("hash", u, num_segs(src, r));
+            PROBE_PRINT("hash", P.rec.u, P.rec.nseg);
             continue;
         }
         // ---- fallback: restore the pairs this row dirtied (each thread its own) --
@@ -732,6 +845,7 @@ hash_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
             for (int sl = 0; sl < 16; ++sl) tabw[sl * MPP + m] = 0xFFFFFFFFu;
             reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
         }
+        pf_commit(N);
         __syncthreads();
     }
 }
@@ -777,7 +891,8 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         for (uint32_t w = 0; w < nwin; ++w) {
             const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseBits;
             const uint64_t whi = min(wlo + kDenseBits, uint64_t(chi) + 1);
-            block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, nullptr, BATCH, [&](idx_t c) {
+            block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH, false,
+                                           [&](idx_t c) {
                 if (c >= wlo && c < whi) {
                     const uint32_t d = uint32_t(c - wlo);
                     const uint32_t bit = 1u << (d & 31);
@@ -878,6 +993,32 @@ __global__ void bin_scatter_kernel(const uint8_t* __restrict__ bin, idx_t nrows,
         __syncthreads();
         if (b > 0) rows[sh_base[b] + local] = idx_t(r);
         __syncthreads();
+    }
+}
+
+// Work records of the hash-bin rows (items [binoff[BIN_H0], binoff[BIN_H6+1])).
+__global__ void make_recs_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ binoff,
+                                 const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
+                                 const uint64_t* __restrict__ soff, RowRec* __restrict__ recs) {
+    const uint32_t lo = binoff[BIN_H0], hi = binoff[BIN_H6 + 1];
+    for (uint32_t i = lo + blockIdx.x * blockDim.x + threadIdx.x; i < hi; i += gridDim.x * blockDim.x) {
+        const idx_t r = rows[i];
+        RowRec x;
+        x.r = r;
+        x.u = uint32_t(min(ub[r], uint64_t(0xFFFFFFFFu)));
+        if (range) {
+            const uint2 rg = range[r];
+            x.clo = rg.x;
+            x.chi = rg.y;
+        } else {
+            x.clo = 0;
+            x.chi = ncols - 1;
+        }
+        x.out = soff[r];
+        x.seg = seg_base(src, r);
+        x.nseg = num_segs(src, r);
+        x.pad = 0;
+        recs[i] = x;
     }
 }
 
@@ -1255,6 +1396,10 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     // the scratch is matrix storage: compacted in place it becomes colidx
     DevBuf<idx_t> scratch(scratch_total, kMat);
     DevBuf<idx_t> ovf_rows(nrows);
+    DevBuf<RowRec> recs(nrows);  // indexed by bin item (only hash-bin items are written)
+    make_recs_kernel<<<gb, 256, 0, st>>>(src, rows.p, binoff, ub, range, ncols, soff.p, recs.p);
+    count_launch();
+    check_launch("make_recs_kernel");
     trace_mark("scratch alloc");
 
     // 4. per-bin kernels, heaviest first, back to back on the library stream
@@ -1267,8 +1412,8 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     ktime_end(t);
 #define LAUNCH_HASH(K, NAME, BIN, W)                                                                  \
     t = ktime_begin(#NAME, st);                                                                         \
-    K<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, rows.p, binoff + BIN, ub, range, ncols, scratch.p, \
-                                                         soff.p, counts.p, work + W, ovf_rows.p, ovf);  \
+    K<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p, counts.p,  \
+                                                         work + W, ovf_rows.p, ovf);                    \
     ktime_end(t);
     LAUNCH_HASH(HASH6, H6, BIN_H6, 7)
     LAUNCH_HASH(HASH5, H5, BIN_H5, 1)
