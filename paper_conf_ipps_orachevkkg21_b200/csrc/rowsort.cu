@@ -1310,7 +1310,7 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
            batch * kSegBytes + first_entries(uint64_t(buckets) * 8) * sizeof(uint32_t) +
            ovcap * (sizeof(idx_t) + sizeof(uint16_t)) + obcap * 2 * sizeof(uint32_t);
 }
-#define HBIN(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U, DB)                                       \
+#define HBIN_(NAME, T, UB, OVCAP, OBCAP, BATCH, PERSM, U, DB)                                       \
     constexpr int NAME##_T = T, NAME##_PERSM = PERSM, NAME##_U = U;                                \
     constexpr bool NAME##_DB = DB;                                                                 \
     constexpr uint32_t NAME##_B = uint32_t(UB / 8), NAME##_OVCAP = OVCAP, NAME##_OBCAP = OBCAP,     \
@@ -1321,13 +1321,35 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
 // <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread,
 //  dedup in pass B (else re-sort in pass A)>
 // (expected per row at mean load 8 with 16 slots: list ~ub/1500, buckets ~ub/2000)
-HBIN(H0, 32, kH0, 32, 16, 64, 32, 4, false)
-HBIN(H1, 64, kH1, 32, 16, 128, 20, 4, false)
-HBIN(H2, 64, kH2, 32, 16, 128, 16, 4, false)
-HBIN(H3, 128, kH3, 64, 32, 256, 8, 4, false)
-HBIN(H4, 256, kH4, 64, 32, 256, 4, 8, true)
-HBIN(H5, 512, kH5, 128, 64, 256, 2, 8, true)
-HBIN(H6, 1024, kH6, 192, 96, 384, 1, 8, true)
+#define HBIN(NAME, ...) HBIN_(NAME, __VA_ARGS__)
+#ifndef H0_CFG  // (overridable for tools/sweep.sh)
+#define H0_CFG 32, kH0, 32, 16, 64, 32, 4, false
+#endif
+HBIN(H0, H0_CFG)
+#ifndef H1_CFG  // (overridable for tools/sweep.sh)
+#define H1_CFG 32, kH1, 32, 16, 128, 24, 4, false
+#endif
+HBIN(H1, H1_CFG)
+#ifndef H2_CFG  // (overridable for tools/sweep.sh)
+#define H2_CFG 64, kH2, 32, 16, 128, 16, 4, false
+#endif
+HBIN(H2, H2_CFG)
+#ifndef H3_CFG  // (overridable for tools/sweep.sh)
+#define H3_CFG 128, kH3, 64, 32, 256, 8, 6, false
+#endif
+HBIN(H3, H3_CFG)
+#ifndef H4_CFG  // (overridable for tools/sweep.sh)
+#define H4_CFG 256, kH4, 64, 32, 256, 4, 6, false
+#endif
+HBIN(H4, H4_CFG)
+#ifndef H5_CFG  // (overridable for tools/sweep.sh)
+#define H5_CFG 512, kH5, 128, 64, 256, 2, 6, false
+#endif
+HBIN(H5, H5_CFG)
+#ifndef H6_CFG  // (overridable for tools/sweep.sh)
+#define H6_CFG 1024, kH6, 192, 96, 384, 1, 4, true
+#endif
+HBIN(H6, H6_CFG)
 #define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U, N##_DB>
 #define HASH0 HASHK(H0)
 #define HASH1 HASHK(H1)
