@@ -638,16 +638,26 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                 uint32_t dsum = 0;
 #pragma unroll
                 for (int k2 = 1; k2 < 16; ++k2) dsum += __vmaxu2(x[k2], vadd2(x[k2 - 1], 0x00010001u)) - x[k2];
-                if (!DEDUP_B && dsum) {  // drop the duplicates here: mark them empty, sort again
-                    uint32_t prev = x[0];
+                if (!DEDUP_B) {
+                    // drop the duplicates here: mark them empty (0xFFFF, the maximum),
+                    // then h bubble passes (adjacent compare-swaps) move the h holes
+                    // of a bucket behind its values; h = the warp's largest
+                    // per-bucket duplicate count (usually 0 or 1)
+                    const uint32_t h = __reduce_max_sync(__activemask(), max(dsum & 0xFFFFu, dsum >> 16));
+                    if (h) {
+                        uint32_t prev = x[0];
 #pragma unroll
-                    for (int k2 = 1; k2 < 16; ++k2) {
-                        const uint32_t cur = x[k2];
-                        x[k2] = cur | ((cur & 0xFFFFu) == (prev & 0xFFFFu) ? 0xFFFFu : 0u) |
-                                ((cur >> 16) == (prev >> 16) ? 0xFFFF0000u : 0u);
-                        prev = cur;
+                        for (int k2 = 1; k2 < 16; ++k2) {
+                            const uint32_t cur = x[k2];
+                            x[k2] = cur | __vcmpeq2(cur, prev);
+                            prev = cur;
+                        }
+#pragma unroll 1
+                        for (uint32_t ps = 0; ps < h; ++ps) {
+#pragma unroll
+                            for (int k2 = 0; k2 < 15; ++k2) cswap2(x[k2], x[k2 + 1]);
+                        }
                     }
-                    sort16x2(x);
                 }
                 if (nn.x <= kSlots) res.x = nn.x - (dsum & 0xFFFFu);
                 if (nn.y <= kSlots) res.y = nn.y - (dsum >> 16);

@@ -18,8 +18,8 @@ for r in csv.reader(io.StringIO(out)):
         try: rows.append((fname, int(r[0]), float(d.get("Instructions Executed", 0) or 0), float(d.get("# Samples", 0) or 0)))
         except ValueError: pass
 k0 = find("hash_bin_kernel(SegSource src")
-marks = [("setup/meta", k0), ("bitmap-mode", find("if (words <= 9ull * nb)", k0)), ("pre-insert", find("PROBE(1);", k0)),
-         ("insert", find("block_products<THREADS, FLATU>(src, r, sd_ptr, sd_end, sd_first, BATCH, [&](idx_t c) {\n", k0) if False else find("const uint32_t b = __umulhi(d, M) >> l;", k0) - 3),
+marks = [("setup/meta", k0), ("bitmap-mode", find("if (P.mode == kPlanBitmap)", k0)), ("pre-insert", find("PROBE(1);", k0)),
+         ("insert", find("const uint32_t b = __umulhi(d, M) >> l;", k0) - 3),
          ("passA", find("// ---- pass A", k0)), ("overflow", find("// ---- overflow buckets", k0)),
          ("scan", find("// ---- multi-scan", k0)), ("passB", find("// ---- pass B", k0)), ("end", find("// ---- fallback: restore", k0))]
 agg = {}
