@@ -9,5 +9,10 @@ timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; cut -c1-200 $O/benc
 timeout 600 python bench.py --impl reference > $O/bench_ref.json 2> $O/bench_ref.err; cut -c1-160 $O/bench_ref.json
 SPBLA_DIST_BACKEND=gloo timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 2 --warmup 3 --workload rmat20_ef16 --no-cpu-baseline > $O/bench_2rank_gloo.json 2> $O/bench_2rank_gloo.err; cut -c1-200 $O/bench_2rank_gloo.json
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_launch_bench.log 2>&1
-timeout 1200 ncu --set full --import-source on --clock-control none -k regex:${TOPK:-hash_bin_kernel} -s ${TOPS:-1} -c 1 -o $O/top python tools/quick_mxm.py 22 32 0.4 0.2 0.2 > $O/ncu_top.log 2>&1
+# ncu --set full of the dominant kernels of one MxM of configs[4] (skip 1 = Build's launch)
+for kv in "compact:compact_inplace" "H4:hash_bin_kernel<.int.256,..unsigned.int.1024," "H5:hash_bin_kernel<.int.512,..unsigned.int.2560,"; do
+  tag=${kv%%:*}; rx=${kv#*:}
+  timeout 900 ncu --set full --import-source on --clock-control none --kernel-name-base demangled -k "regex:$rx" -s 1 -c 1 \
+     -o $O/top_$tag -f python tools/quick_mxm.py 22 32 0.4 0.2 0.2 5 > $O/ncu_top_$tag.log 2>&1
+done
 ls -la $O

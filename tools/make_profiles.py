@@ -20,8 +20,8 @@ for r in rows[hi + 1:]:
     v *= {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3}.get(r[ui], 1.0)
     m = re.search(r'(\w+_kernel)(<[^>]*>)?', name)
     seq.append(((m.group(1) + (m.group(2) or '')) if m else name[:60], v, 'spbla' in name))
-# last step = from the last mxm_ub_kernel to the end
-last = max(i for i, s in enumerate(seq) if s[0].startswith('mxm_ub_kernel'))
+# last step = from the last row_span_kernel (first launch of an MxM) to the end
+last = max(i for i, s in enumerate(seq) if s[0].startswith('row_span_kernel'))
 step = [s for s in seq[last:] if s[2]]
 tot = sum(v for _, v, _ in step)
 out.append(f"# {tag}: ncu launch list of one bench.py step (configs[4], rmat22_ef32 A.A)\n")
@@ -32,17 +32,20 @@ for name, v, _ in step:
     out.append(f"| `{name}` | {v:.1f} | {v / tot * 100:.1f}% |")
 out.append(f"| **total (library kernels)** | {tot:.1f} | 100% |\n")
 
-# 2. full capture of the top kernel
-rep = os.path.join(CK, "top.ncu-rep")
+# 2. full captures of the dominant kernels (top_<group>.ncu-rep)
+import glob
 traffic = {}
-if os.path.exists(rep):
+for rep in sorted(glob.glob(os.path.join(CK, "top_*.ncu-rep"))):
+    grp = os.path.basename(rep)[4:-8]
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rr = list(csv.reader(io.StringIO(raw)))
+    if len(rr) < 3:
+        continue
     hh, uu, vv = rr[0], rr[1], rr[2]
     def g(k):
         return (vv[hh.index(k)], uu[hh.index(k)]) if k in hh else ("n/a", "")
     kname = vv[hh.index("Kernel Name")]
-    out.append(f"## ncu --set full: `{kname[:110]}`\n")
+    out.append(f"## ncu --set full ({grp}): `{kname[:110]}`\n")
     keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
             "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed",
             "dram__throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
@@ -57,12 +60,12 @@ if os.path.exists(rep):
               if 'pcsamp_warps_issue_stalled' in hh[i] and not hh[i].endswith('not_issued')]
     st = sum(s for _, s in stalls) or 1
     out.append("\nWarp-state samples (top):\n")
-    for n, s in sorted(stalls, key=lambda x: -x[1])[:6]:
-        out.append(f"- {n.replace('smsp__pcsamp_warps_issue_stalled_', '')}: {s / st * 100:.1f}%")
-    rd = float(g("dram__bytes_read.sum")[0]); wr = float(g("dram__bytes_write.sum")[0])
-    unit = g("dram__bytes_read.sum")[1]
-    scale = {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}.get(unit, 1)
-    traffic = {"kernel": kname[:120], "dram_bytes_per_launch": (rd + wr) * scale}
+    for nm, sv in sorted(stalls, key=lambda x: -x[1])[:6]:
+        out.append(f"- {nm.replace('smsp__pcsamp_warps_issue_stalled_', '')}: {sv / st * 100:.1f}%")
+    def gb(k):
+        val, un = g(k)
+        return float(val) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}.get(un, 1)
+    traffic[grp] = (gb("dram__bytes_read.sum") + gb("dram__bytes_write.sum"), kname)
     out.append("")
 
 # 3. bench lines
@@ -74,8 +77,8 @@ open(os.path.join(P, f"{tag}_summary.md"), "w").write("\n".join(out) + "\n")
 if traffic:
     tp = os.path.join(P, "ncu_traffic.json")
     tj = json.load(open(tp)) if os.path.exists(tp) else {}
-    grp = os.environ.get("TOP_GROUP", "H5")
-    tj.setdefault("rmat22_ef32", {})[grp] = traffic["dram_bytes_per_launch"]
-    tj.setdefault("_source", {})[grp] = f"profiles/{tag}_summary.md: {traffic['kernel'][:80]}"
+    for grp, (byt, kname) in traffic.items():
+        tj.setdefault("rmat22_ef32", {})[grp] = byt
+        tj.setdefault("_source", {})[grp] = f"profiles/{tag}_summary.md: {kname[:80]}"
     json.dump(tj, open(tp, "w"), indent=1)
 print(open(os.path.join(P, f"{tag}_summary.md")).read()[:3000])
