@@ -37,6 +37,9 @@ WORKLOADS = {
     "uniform4096": dict(config="configs[0]", scale=12, ef=8, abc=None, seed=1),
 }
 DEFAULT_WORKLOAD = "rmat22_ef32"
+# the other BASELINE.json rows (own metric lines, not the headline): configs[2]
+# EWiseAdd + Kronecker, configs[3] transitive closure
+AUX_WORKLOADS = ("ewise_kron", "closure18")
 FLUSH_BYTES = 256 << 20
 
 
@@ -174,17 +177,123 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+
+# ---------------------------------------------------------------------------
+def run_aux(args):
+    """configs[2] (EWiseAdd 2^20 rows, Kronecker 2^10 graph x 64-state RSM) and
+    configs[3] (closure of a 2^18-vertex labelled DAG): device-timed with CUDA
+    events on the library stream, L2 flushed between steps; one JSON line.
+    1 GPU (these rows are replicas-only at N > 1)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import paper_conf_ipps_orachevkkg21_b200 as sp
+    torch.cuda.set_device(0)
+    sp.Initialize(0)
+    stream = torch.cuda.current_stream()
+    peak_gbs, peak_src = load_peaks()
+    flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device="cuda")
+    steps, warmup = args.steps, max(args.warmup, 3)
+    launches = []
+
+    def timed(fn):
+        for _ in range(warmup):
+            fn()
+        torch.cuda.synchronize()
+        sp.set_kernel_timing(True)
+        sp.reset_launch_count()
+        ms = []
+        for _ in range(steps):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            fn()
+            e1.record(stream)
+            e1.synchronize()
+            ms.append(e0.elapsed_time(e1))
+        launches.append(sp.launch_count())
+        return sum(ms) / len(ms)
+
+    clocks = ClockSampler(0)
+    if args.workload == "ewise_kron":
+        n = 1 << 20
+        r1, c1 = spgen.rmat_pairs(20, 16, 0.45, 0.22, 0.22, seed=1, device="cuda")
+        r2, c2 = spgen.uniform_pairs(n, n, 8, seed=2, device="cuda")
+        A = sp.Matrix.from_pairs(n, n, r1, c1)
+        B = sp.Matrix.from_pairs(n, n, r2, c2)
+        E = sp.Matrix.new(n, n)
+        ms_e = timed(lambda: sp.Matrix_EWiseAdd(E, A, B))
+        ke = {k: sp.kernel_timing(k) for k in ("ewise_split", "ewise_merge")}
+        sp.set_kernel_timing(False)
+        # algorithmic bytes: both inputs read once (colidx + rowptr), output written once
+        alg_e = 4 * (A.nvals + B.nvals) + 16 * (n + 1) + 4 * E.nvals + 8 * (n + 1)
+        rg, cg = spgen.rmat_pairs(10, 16, 0.45, 0.22, 0.22, seed=3, device="cuda")
+        rr, cr = spgen.rsm_pairs(64, 1, 2, seed=4, device="cuda")
+        G = sp.Matrix.from_pairs(1024, 1024, rg, cg)
+        R = sp.Matrix.from_pairs(64, 64, rr, cr)
+        K = sp.Matrix.new(1024 * 64, 1024 * 64)
+        ms_k = timed(lambda: sp.Kronecker(K, G, R))
+        kk = sp.kernel_timing("kron")
+        sp.set_kernel_timing(False)
+        alg_k = 4 * K.nvals + 8 * (K.nrows + 1)  # output-write bound (inputs are KB)
+        clk = clocks.stop()
+        per_e = (ke["ewise_split"][0] + ke["ewise_merge"][0]) / steps
+        line = {"metric": "configs[2] EWiseAdd (2^20 rows) + Kronecker (2^10 x 64-state RSM): ms, GB/s vs HBM peak",
+                "value": ms_e + ms_k, "unit": "ms", "higher_is_better": False, "n_gpus": 1, "steps": steps,
+                "warmup": warmup, "dtype": "u32", "data": "synthetic (DESIGN.md §3)",
+                "config": {"workload": "ewise_kron", "baseline_config": "configs[2]",
+                           "l2": "256 MB write between timed steps"},
+                "ewise": {"ms": ms_e, "kernel_ms": per_e, "nnz_A": A.nvals, "nnz_B": B.nvals, "nnz_C": E.nvals,
+                          "alg_bytes": alg_e, "GB/s": alg_e / (per_e * 1e-3) / 1e9,
+                          "frac": alg_e / (per_e * 1e-3) / 1e9 / peak_gbs,
+                          "kernel_ms_per_step": {k: v[0] / steps for k, v in ke.items()}},
+                "kron": {"ms": ms_k, "kernel_ms": kk[0] / steps, "nnz_K": K.nvals, "rows_K": K.nrows,
+                         "alg_bytes": alg_k, "GB/s": alg_k / (kk[0] / steps * 1e-3) / 1e9,
+                         "frac": alg_k / (kk[0] / steps * 1e-3) / 1e9 / peak_gbs},
+                "peak": peak_gbs, "peak_source": peak_src, "clocks": clk}
+    else:
+        n = 1 << 18
+        (a0, b0), (a1, b1) = spgen.labeled_dag(n, 0.25, seed=9, device="cuda")
+        L0 = sp.Matrix.from_pairs(n, n, a0, b0)
+        L1 = sp.Matrix.from_pairs(n, n, a1, b1)
+        U = sp.ewise_add(L0, L1)
+        state = {}
+
+        def step():
+            C = U.duplicate()
+            state["it"] = sp.TransitiveClosure(C)
+            state["nnz"] = C.nvals
+            C.free()
+        ms_c = timed(step)
+        groups = ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "compact")
+        kt = {k: sp.kernel_timing(k)[0] / steps for k in groups}
+        sp.set_kernel_timing(False)
+        clk = clocks.stop()
+        line = {"metric": "configs[3] transitive closure C += C.C to fixed point (2^18-vertex labelled DAG): ms",
+                "value": ms_c, "unit": "ms", "higher_is_better": False, "n_gpus": 1, "steps": steps,
+                "warmup": warmup, "dtype": "u32", "data": "synthetic (DESIGN.md §3)",
+                "config": {"workload": "closure18", "baseline_config": "configs[3]", "vertices": n,
+                           "nnz_in": U.nvals, "nnz_closure": state["nnz"], "iterations": state["it"],
+                           "l2": "256 MB write between timed steps"},
+                "ms_per_iteration": ms_c / state["it"], "kernel_ms_per_step": kt, "clocks": clk}
+    line["gpu_launches"] = sum(launches)
+    print(json.dumps(line), flush=True)
+
+
 # ---------------------------------------------------------------------------
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--workload", default=DEFAULT_WORKLOAD, choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default=DEFAULT_WORKLOAD, choices=sorted(WORKLOADS) + list(AUX_WORKLOADS))
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
+    if args.workload in AUX_WORKLOADS:
+        return run_aux(args)
     if args.impl == "reference":
         return run_reference(args)
     args.warmup = max(args.warmup, 3)

@@ -1,19 +1,26 @@
 // Element-wise addition C = A + B (§III-A l.266-269: "GPU
 // Merge Path algorithm with dynamic work balancing and two pass processing").
 //
-// The two CSR matrices are treated as two sorted sequences of (row, col)
-// keys; their merge (ties: A first) is the row-major concatenation of the
-// per-row merges, and row r starts at merged position p(r) = rpA[r] + rpB[r].
-// Merge path cuts the merged sequence into equal tiles of kTile items, so
-// every thread gets exactly kItems merged items whatever the row-length
-// skew.  A B item is a duplicate iff the A item just before it in its row
-// has the same column (rows are sorted and duplicate-free).  Output position
-// of a kept item at merged position d is d - (#duplicates before d), and
-// rowptrC[r] = p(r) - (#duplicates before p(r)).
-//   pass 1: duplicates per tile  -> in-house scan -> nnz(C)
-//   pass 2: same merge, block scan of per-thread duplicates, write colidx and
-//           the row offsets of rows starting inside the thread's range.
-// HBM bytes (algorithmic): 2 x 4(nnzA + nnzB) read + 4 nnz(C) + 8(m+1) written.
+// The two CSR matrices are two sorted sequences of (row, col) keys; their
+// merge (ties: A first) is the row-major concatenation of the per-row merges,
+// and row r starts at merged position P(r) = rpA[r] + rpB[r].  Merge path cuts
+// the merged sequence into equal tiles of kTile items, so every block gets
+// exactly kTile merged items whatever the row-length skew.  A B item is a
+// duplicate iff the merged item just before it is the A item with the same
+// key (rows are sorted and duplicate-free).
+//
+// B200 design: ONE pass over the inputs instead of the paper's two.
+//   ewise_split_kernel : per row, the merge-path split (A count) of every
+//                        tile boundary inside the row, and for every tile the
+//                        first row whose merged start lies in it.
+//   ewise_merge_kernel : per tile (ticket order): coalesced staging of the
+//                        tile's A and B ranges as 64-bit (row, col) keys in
+//                        shared memory, merge path per thread in smem, block
+//                        scan of duplicates, decoupled look-back over the
+//                        tiles' kept counts for the output base, coalesced
+//                        writes of colidx through smem, and the row offsets
+//                        of the rows starting in the tile.
+// HBM bytes: 4(nnzA + nnzB) + 16(m+1) read, 4 nnz(C) + 8(m+1) written.
 #include "common.cuh"
 
 #include <algorithm>
@@ -22,9 +29,20 @@ namespace spbla {
 
 namespace {
 
-constexpr int kThreads = 128;
-constexpr int kItems = 16;
-constexpr int kTile = kThreads * kItems;
+constexpr int kThreads = 256;
+constexpr int kItems = 8;
+constexpr uint32_t kTile = kThreads * kItems;  // 2048 merged items per tile
+// padded smem indices: threads own kItems consecutive positions, so a plain
+// layout puts the lanes of a warp kItems words apart (8- to 16-way bank
+// conflicts); one pad word per 16 (keys, 64-bit) / 32 (marks, output) words
+// spreads them over all banks
+__device__ __forceinline__ uint32_t KI(uint32_t p) { return p + (p >> 4); }
+__device__ __forceinline__ uint32_t OI(uint32_t p) { return p + (p >> 5); }
+constexpr uint32_t kKeyWords = kTile + kTile / 16, kOutWords = kTile + kTile / 32 + 1;
+constexpr size_t kMergeSmem = size_t(kKeyWords) * 8 + size_t(kOutWords) * 4 + (kTile + 1) * 2;
+constexpr uint64_t kFlagAgg = 1ull << 62;
+constexpr uint64_t kFlagPre = 2ull << 62;
+constexpr uint64_t kValMask = (1ull << 62) - 1;
 
 struct MergeIn {
     idx_t nrows;
@@ -32,147 +50,219 @@ struct MergeIn {
     const idx_t* __restrict__ ca;
     const off_t64* __restrict__ rpb;
     const idx_t* __restrict__ cb;
-    uint64_t L;
+    uint64_t L;  // nnzA + nnzB
 };
 
 __device__ __forceinline__ uint64_t P(const MergeIn& m, idx_t r) { return m.rpa[r] + m.rpb[r]; }
 
-// first row r in [lo, hi] with P(r) >= d (hi if none)
-__device__ __forceinline__ idx_t rows_lower_bound(const MergeIn& m, idx_t lo, idx_t hi, uint64_t d) {
-    while (lo < hi) {
-        idx_t mid = lo + (hi - lo) / 2;
-        if (P(m, mid) < d) lo = mid + 1; else hi = mid;
+// Per row r: for every tile boundary d = t*kTile in [P(r), P(r+1)) (non-empty
+// rows only), tile_row[t] = r and tile_a[t] = the A position of the
+// merge-path split of the row's first q = d - P(r) merged items (ties: A
+// first); for every tile t with P(r-1) < t*kTile <= P(r), tile_rlo[t] = r
+// (the first row whose merged start is in tile t or later).  The sentinel
+// tile_row / tile_a[ntiles] is written by row nrows.  tile_prev[t]: the key
+// of the A item just before the split if it lies in the same row.
+__global__ void ewise_split_kernel(MergeIn m, uint64_t ntiles, uint32_t* __restrict__ tile_row,
+                                   uint64_t* __restrict__ tile_a, uint32_t* __restrict__ tile_rlo,
+                                   uint64_t* __restrict__ tile_prev) {
+    for (size_t r = blockIdx.x * size_t(blockDim.x) + threadIdx.x; r <= m.nrows; r += size_t(gridDim.x) * blockDim.x) {
+        const uint64_t p = P(m, idx_t(r));
+        const uint64_t pprev = r ? P(m, idx_t(r - 1)) : 0;
+        for (uint64_t t = r ? pprev / kTile + 1 : 0; t * kTile <= p && t <= ntiles; ++t) tile_rlo[t] = uint32_t(r);
+        if (r == m.nrows) {
+            tile_row[ntiles] = m.nrows;
+            tile_a[ntiles] = m.rpa[m.nrows];
+            continue;
+        }
+        const uint64_t sa = m.rpa[r], sb = m.rpb[r];
+        const uint64_t la = m.rpa[r + 1] - sa, lb = m.rpb[r + 1] - sb;
+        for (uint64_t t = (p + kTile - 1) / kTile; t * kTile < p + la + lb; ++t) {
+            const uint64_t q = t * kTile - p;
+            uint64_t lo = q > lb ? q - lb : 0, hi = q < la ? q : la;
+            while (lo < hi) {
+                const uint64_t mid = (lo + hi) >> 1;
+                if (m.ca[sa + mid] <= m.cb[sb + q - 1 - mid]) lo = mid + 1; else hi = mid;
+            }
+            tile_row[t] = uint32_t(r);
+            tile_a[t] = sa + lo;
+            // the A item just before the split as a key: only an item of the
+            // same row can equal a B key of tile t
+            tile_prev[t] = lo > 0 ? ((uint64_t(r) << 32) | m.ca[sa + lo - 1]) : ~0ull;
+        }
     }
-    return lo;
-}
-// first row r in [lo, hi] with P(r) > d
-__device__ __forceinline__ idx_t rows_upper_bound(const MergeIn& m, idx_t lo, idx_t hi, uint64_t d) {
-    while (lo < hi) {
-        idx_t mid = lo + (hi - lo) / 2;
-        if (P(m, mid) <= d) lo = mid + 1; else hi = mid;
-    }
-    return lo;
-}
-
-struct Cursor {
-    idx_t r;        // current row
-    uint64_t a, b;  // global positions in A / B colidx
-    uint64_t ea, eb, sa;  // row end in A, end in B, row start in A
-};
-
-// Position the cursor at merged position d < L (row search within [rlo, rhi]).
-__device__ __forceinline__ Cursor locate(const MergeIn& m, uint64_t d, idx_t rlo, idx_t rhi) {
-    Cursor c;
-    c.r = rows_upper_bound(m, rlo, rhi, d) - 1;  // largest r with P(r) <= d
-    const uint64_t sa = m.rpa[c.r], sb = m.rpb[c.r];
-    const uint64_t la = m.rpa[c.r + 1] - sa, lb = m.rpb[c.r + 1] - sb;
-    const uint64_t q = d - (sa + sb);
-    uint64_t lo = q > lb ? q - lb : 0, hi = q < la ? q : la;
-    while (lo < hi) {
-        uint64_t mid = (lo + hi) >> 1;
-        if (m.ca[sa + mid] <= m.cb[sb + q - 1 - mid]) lo = mid + 1; else hi = mid;
-    }
-    c.a = sa + lo;
-    c.b = sb + (q - lo);
-    c.sa = sa;
-    c.ea = sa + la;
-    c.eb = sb + lb;
-    return c;
 }
 
-// Take the next merged item; returns its column and whether it duplicates
-// the previous A item of the same row.
-__device__ __forceinline__ idx_t take(const MergeIn& m, Cursor& c, bool& dup) {
-    while (c.a == c.ea && c.b == c.eb) {  // row exhausted: advance (skips empty rows)
-        ++c.r;
-        c.sa = c.ea;
-        c.ea = m.rpa[c.r + 1];
-        c.eb = m.rpb[c.r + 1];
-    }
-    if (c.a < c.ea && (c.b == c.eb || m.ca[c.a] <= m.cb[c.b])) {
-        dup = false;
-        return m.ca[c.a++];
-    }
-    idx_t v = m.cb[c.b++];
-    dup = (c.a > c.sa) && (m.ca[c.a - 1] == v);
+__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 
-__device__ __forceinline__ void tile_rows(const MergeIn& m, uint64_t d0, uint64_t d1, idx_t* sr) {
-    if (threadIdx.x == 0) {
-        // one row before the first row starting at or after d0, so that empty
-        // rows starting exactly at d0 are inside [sr0, sr1]
-        idx_t lo = rows_lower_bound(m, 0, m.nrows, d0);
-        sr[0] = lo > 0 ? lo - 1 : 0;
-        sr[1] = rows_upper_bound(m, sr[0], m.nrows, d1);
-    }
+__global__ void __launch_bounds__(kThreads, 6)
+ewise_merge_kernel(MergeIn m, uint64_t ntiles, const uint32_t* __restrict__ tile_row,
+                   const uint64_t* __restrict__ tile_a, const uint32_t* __restrict__ tile_rlo,
+                   const uint64_t* __restrict__ tile_prev, uint64_t* status, uint32_t* ticket,
+                   idx_t* __restrict__ out, off_t64* __restrict__ rowptr) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    uint64_t* s_key = reinterpret_cast<uint64_t*>(smem_raw);    // [kTile] A keys [0, na), B keys [na, len)
+    uint32_t* s_out = reinterpret_cast<uint32_t*>(s_key + kKeyWords);  // kept columns in output order (OI)
+    uint16_t* s_dpre = reinterpret_cast<uint16_t*>(s_out + kOutWords);  // [kTile+1] duplicates before each position
+    __shared__ uint64_t sh[33];
+    __shared__ uint32_t s_t;
+    __shared__ uint64_t s_base;
+    uint32_t* s_mark = s_out;  // row marks (scratch until the output is staged)
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) s_mark[OI(threadIdx.x * kItems + k)] = 0u;
+    if (threadIdx.x == 0) s_t = atomicAdd(ticket, 1u);  // ticket order: the look-back never waits on a later block
     __syncthreads();
-}
-
-__global__ void __launch_bounds__(kThreads) merge_count_kernel(MergeIn m, uint64_t* __restrict__ tile_dups) {
-    __shared__ idx_t sr[2];
-    __shared__ uint32_t swarp[kThreads / 32];
-    const uint64_t d0 = uint64_t(blockIdx.x) * kTile;
-    const uint64_t d1 = min(d0 + kTile, m.L);
-    tile_rows(m, d0, d1, sr);
-    const uint64_t db = d0 + uint64_t(threadIdx.x) * kItems;
-    uint32_t dups = 0;
-    if (db < d1) {
-        Cursor c = locate(m, db, sr[0], sr[1]);
-        const uint64_t de = min(db + kItems, d1);
-        for (uint64_t d = db; d < de; ++d) {
-            bool dup;
-            take(m, c, dup);
-            dups += dup;
+    const uint64_t t = s_t;
+    const uint64_t d0 = t * kTile, d1 = min(d0 + kTile, m.L);
+    const uint32_t len = uint32_t(d1 - d0);
+    const uint64_t a0 = tile_a[t], a1 = tile_a[t + 1];
+    const uint64_t b0 = d0 - a0, b1 = d1 - a1;
+    const uint32_t na = uint32_t(a1 - a0), nb = uint32_t(b1 - b0);
+    const uint32_t r0 = tile_row[t], r1 = min(tile_row[t + 1], m.nrows - 1);
+    const uint64_t prevA = tile_prev[t];
+    // 1. stage the columns (coalesced) and, in the same round trip, mark the
+    //    first tile position of every row segment (0 = no mark; B marks are
+    //    offset by nrows + 1 so that no A row carries into the B part); a
+    //    max-scan then gives every position its row, ORed into the key
+    {
+        idx_t cv[kItems];  // all loads in flight before the first smem store
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            const uint32_t pos = k * kThreads + threadIdx.x;
+            cv[k] = pos < na ? m.ca[a0 + pos] : (pos < len ? m.cb[b0 + (pos - na)] : 0u);
+        }
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            const uint32_t pos = k * kThreads + threadIdx.x;
+            if (pos < len) s_key[KI(pos)] = cv[k];
         }
     }
-    dups = warp_sum(dups);
-    if (lane_id() == 0) swarp[threadIdx.x >> 5] = dups;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        uint64_t s = 0;
-        for (int w = 0; w < kThreads / 32; ++w) s += swarp[w];
-        tile_dups[blockIdx.x] = s;
+    const uint32_t boff = m.nrows + 1;
+#pragma unroll 1
+    for (uint32_t r = r0 + threadIdx.x; r <= r1; r += kThreads) {
+        const uint64_t ra = max(m.rpa[r], a0), rae = min(m.rpa[r + 1], a1);
+        const uint64_t rb = max(m.rpb[r], b0), rbe = min(m.rpb[r + 1], b1);
+        if (ra < rae) s_mark[OI(uint32_t(ra - a0))] = r + 1;
+        if (rb < rbe) s_mark[OI(na + uint32_t(rb - b0))] = boff + r + 1;
     }
-}
-
-__global__ void __launch_bounds__(kThreads)
-merge_write_kernel(MergeIn m, const uint64_t* __restrict__ tile_base, idx_t* __restrict__ out,
-                   off_t64* __restrict__ rowptr) {
-    __shared__ idx_t sr[2];
-    __shared__ uint64_t shs[33];
-    const uint64_t d0 = uint64_t(blockIdx.x) * kTile;
-    const uint64_t d1 = min(d0 + kTile, m.L);
-    tile_rows(m, d0, d1, sr);
-    const uint64_t db = d0 + uint64_t(threadIdx.x) * kItems;
-    const uint64_t de = min(db + kItems, d1);
-    // pass A: this thread's duplicate count (re-merge; cheap, data in L1)
-    uint64_t mydups = 0;
-    Cursor c0;
-    if (db < d1) {
-        c0 = locate(m, db, sr[0], sr[1]);
-        Cursor c = c0;
-        for (uint64_t d = db; d < de; ++d) {
-            bool dup;
-            take(m, c, dup);
-            mydups += dup;
+    __syncthreads();
+    {
+        uint32_t v[kItems], run = 0;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            run = max(run, s_mark[OI(threadIdx.x * kItems + k)]);
+            v[k] = run;
+        }
+        // block exclusive max-scan of the thread maxima
+        uint32_t inc = run;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, d);
+            if (int(lane_id()) >= d) inc = max(inc, y);
+        }
+        __shared__ uint32_t s_wmax[kThreads / 32];
+        if (lane_id() == 31) s_wmax[threadIdx.x >> 5] = inc;
+        __syncthreads();
+        uint32_t carry = 0;
+        for (unsigned w = 0; w < (threadIdx.x >> 5); ++w) carry = max(carry, s_wmax[w]);
+        const uint32_t ex = max(carry, __shfl_up_sync(0xffffffffu, inc, 1) * (lane_id() > 0));
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            const uint32_t pos = threadIdx.x * kItems + k;
+            if (pos < len) {
+                uint32_t rr = max(ex, v[k]) - 1;
+                if (pos >= na) rr -= boff;
+                s_key[KI(pos)] |= uint64_t(rr) << 32;
+            }
         }
     }
-    uint64_t tot;
-    uint64_t before = tile_base[blockIdx.x] + block_exclusive_scan<uint64_t>(mydups, shs, &tot);
-    if (db >= d1) return;
-    // rows whose merged start lies in [db, de) (including empty rows)
-    idx_t nr = rows_lower_bound(m, sr[0], sr[1], db);
-    Cursor c = c0;
-    for (uint64_t d = db; d < de; ++d) {
-        while (nr < m.nrows && P(m, nr) == d) rowptr[nr++] = d - before;
-        bool dup;
-        idx_t v = take(m, c, dup);
-        if (dup) ++before;
-        else out[d - before] = v;
+    __syncthreads();
+    // 2. merge path per thread over the smem keys, kItems items each
+    const uint32_t k0 = min(uint32_t(threadIdx.x) * kItems, len), k1 = min(k0 + kItems, len);
+    uint32_t lo = k0 > nb ? k0 - nb : 0, hi = min(k0, na);
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_key[KI(mid)] <= s_key[KI(na + k0 - 1 - mid)]) lo = mid + 1; else hi = mid;
     }
-    if (de == m.L) {  // trailing empty rows and rowptr[nrows]
-        while (nr <= m.nrows && P(m, nr) == m.L) rowptr[nr++] = m.L - before;
+    uint32_t ai = lo, bi = k0 - lo;
+    idx_t col[kItems];
+    uint32_t dmask = 0, ndup = 0;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+        col[k] = 0;
+        if (k0 + k < k1) {
+            const bool takeA = ai < na && (bi == nb || s_key[KI(ai)] <= s_key[KI(na + bi)]);
+            if (takeA) {
+                col[k] = idx_t(s_key[KI(ai++)]);
+            } else {
+                const uint64_t kb = s_key[KI(na + bi++)];
+                const uint64_t pa = ai > 0 ? s_key[KI(ai - 1)] : prevA;
+                col[k] = idx_t(kb);
+                if (pa == kb) {
+                    dmask |= 1u << k;
+                    ++ndup;
+                }
+            }
+        }
+    }
+    // 3. duplicates before every tile position; the tile's kept count
+    uint64_t tdup;
+    const uint32_t dex = uint32_t(block_exclusive_scan<uint64_t>(ndup, sh, &tdup));
+    {
+        uint32_t run = dex;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            if (k0 + k < k1) s_dpre[k0 + k] = uint16_t(run);
+            run += (dmask >> k) & 1u;
+        }
+        if (k1 == len && k0 < k1) s_dpre[len] = uint16_t(run);
+    }
+    const uint64_t kept = len - tdup;
+    // 4. decoupled look-back over the tiles' kept counts, one warp reading a
+    //    window of 32 predecessors per round trip (a serial one-tile-per-load
+    //    look-back falls behind the tiles in flight and serialises the grid)
+    if (threadIdx.x < 32) {
+        const unsigned lane = lane_id();
+        uint64_t prefix = 0;
+        if (t == 0) {
+            if (lane == 0) st_relaxed(&status[0], kFlagPre | kept);
+        } else {
+            if (lane == 0) st_relaxed(&status[t], kFlagAgg | kept);
+            for (long j = long(t) - 1;; j -= 32) {
+                const long idx = j - long(lane);  // lane 0 = the nearest predecessor
+                uint64_t s = idx >= 0 ? ld_relaxed(&status[idx]) : kFlagPre;
+                while (__any_sync(0xffffffffu, (s >> 62) == 0))
+                    if ((s >> 62) == 0) s = ld_relaxed(&status[idx]);
+                const uint32_t pre = __ballot_sync(0xffffffffu, (s >> 62) == 2);
+                const int first = pre ? __ffs(pre) - 1 : 31;
+                prefix += warp_sum(int(lane) <= first ? (s & kValMask) : 0ull);
+                if (pre) break;
+            }
+            if (lane == 0) st_relaxed(&status[t], kFlagPre | (prefix + kept));
+        }
+        if (lane == 0) s_base = prefix;
+    }
+    // 5. kept columns to smem in output order, then coalesced stores
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+        const uint32_t pos = k0 + k;
+        if (pos < k1 && !((dmask >> k) & 1u)) s_out[OI(pos - s_dpre[pos])] = col[k];
+    }
+    __syncthreads();
+    const uint64_t base = s_base;
+    for (uint32_t i = threadIdx.x; i < kept; i += kThreads) out[base + i] = s_out[OI(i)];
+    // 6. row offsets of the rows starting in [d0, d1); the last tile also
+    //    writes the rows starting at L (trailing empty rows, rowptr[nrows])
+    const uint32_t rlo = tile_rlo[t], rhi = (t + 1 == ntiles) ? m.nrows + 1 : tile_rlo[t + 1];
+    for (uint32_t r = rlo + threadIdx.x; r < rhi; r += kThreads) {
+        const uint32_t p = uint32_t(P(m, r) - d0);
+        rowptr[r] = base + p - s_dpre[p];
     }
 }
 
@@ -188,20 +278,37 @@ void ewise_add(Matrix* C, const Matrix* A, const Matrix* B) {
         return;
     }
     const uint64_t ntiles = ceil_div(m.L, kTile);
-    DevBuf<uint64_t> tdup(ntiles);
-    DevBuf<uint64_t> tbase(ntiles + 1);
-    merge_count_kernel<<<(unsigned)ntiles, kThreads, 0, ctx().stream>>>(m, tdup.p);
-    count_launch();
-    check_launch("merge_count_kernel");
-    exclusive_scan_u64(tdup.p, tbase.p, ntiles);
-    uint64_t h;
-    read_words(tbase.p + ntiles, &h, 1);
-    const uint64_t nnz = m.L - h;
+    const int nsm = ctx().num_sms;
+    // tile_row[ntiles+1] | tile_rlo[ntiles+1] (u32), tile_a[ntiles+1] | tile_prev[ntiles+1],
+    // status[ntiles] + ticket
+    DevBuf<uint32_t> trow(2 * (ntiles + 1));
+    DevBuf<uint64_t> ta(2 * (ntiles + 1));
+    DevBuf<uint64_t> status(ntiles + 1);
+    memset_async(status.p, 0, status.n * sizeof(uint64_t));
+    // the result: colidx capacity nnzA + nnzB (>= nnz(C)); the exact nnz is read back
     DevBuf<off_t64> rp(size_t(A->nrows) + 1, kMat);
-    DevBuf<idx_t> ci(nnz, kMat);
-    merge_write_kernel<<<(unsigned)ntiles, kThreads, 0, ctx().stream>>>(m, tbase.p, ci.p, rp.p);
+    DevBuf<idx_t> ci(m.L, kMat);
+    int t = ktime_begin("ewise_split", ctx().stream);
+    const unsigned g1 = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(A->nrows) + 1, 256), uint64_t(nsm) * 8);
+    ewise_split_kernel<<<g1, 256, 0, ctx().stream>>>(m, ntiles, trow.p, ta.p, trow.p + ntiles + 1, ta.p + ntiles + 1);
+    ktime_end(t);
     count_launch();
-    check_launch("merge_write_kernel");
+    check_launch("ewise_split_kernel");
+    static int attr_dev = -1;
+    if (attr_dev != ctx().device) {
+        CUDA_CHECK(cudaFuncSetAttribute(ewise_merge_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kMergeSmem)));
+        attr_dev = ctx().device;
+    }
+    t = ktime_begin("ewise_merge", ctx().stream);
+    ewise_merge_kernel<<<(unsigned)ntiles, kThreads, kMergeSmem, ctx().stream>>>(
+        m, ntiles, trow.p, ta.p, trow.p + ntiles + 1, ta.p + ntiles + 1, status.p,
+        reinterpret_cast<uint32_t*>(status.p + ntiles),
+        ci.p, rp.p);
+    ktime_end(t);
+    count_launch();
+    check_launch("ewise_merge_kernel");
+    uint64_t nnz;
+    read_words(rp.p + A->nrows, &nnz, 1);
     size_t rc = rp.n, cc = ci.n;
     matrix_replace(C, rp.detach(), rc, ci.detach(), cc, nnz);
 }

@@ -60,6 +60,7 @@ void kronecker(Matrix* K, const Matrix* A, const Matrix* B) {
     DevBuf<idx_t> ci(nnz, kMat);
     const int nsm = ctx().num_sms;
     unsigned g1 = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(m + 1, 256), uint64_t(nsm) * 16));
+    const int t = ktime_begin("kron", ctx().stream);
     kron_rowptr_kernel<<<g1, 256, 0, ctx().stream>>>(view(A), view(B), B->nnz, rp.p);
     count_launch();
     check_launch("kron_rowptr_kernel");
@@ -69,6 +70,7 @@ void kronecker(Matrix* K, const Matrix* A, const Matrix* B) {
         count_launch();
         check_launch("kron_cols_kernel");
     }
+    ktime_end(t);
     size_t rc = rp.n, cc = ci.n;
     matrix_replace(K, rp.detach(), rc, ci.detach(), cc, nnz);
 }
