@@ -72,7 +72,7 @@ enum {
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 // hash bins: ub limits (each sized so its tables fit the residency below)
 constexpr uint64_t kH0 = 512, kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480, kH6 = 40960;
-constexpr uint32_t kDenseBits = 1u << 20;      // bitmap window: 128 KB of smem
+constexpr uint32_t kDenseBits = 3u << 19;      // bitmap window: 1.5 Mi columns, 192 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
 __device__ __forceinline__ int bin_of(uint64_t ub) {
@@ -1313,7 +1313,7 @@ constexpr size_t kSegBytes = sizeof(void*) + sizeof(uint32_t);
 // hash bins: <threads, max buckets (= ub limit / 4), overflow slots, descriptor
 // batch, blocks per SM, loads in flight>; smem per block is checked against
 // the residency so each bin keeps its blocks/SM (register-limited at 40 regs)
-constexpr uint32_t kDBatch = 2048;
+constexpr uint32_t kDBatch = 1024;
 constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, uint32_t ovcap, uint32_t obcap) {
     return size_t(16) * pair_stride(buckets / 2) * sizeof(uint32_t) +          // table
            buckets * sizeof(uint32_t) + (buckets / 2) * sizeof(uint32_t) +     // counters, pair offsets
@@ -1369,6 +1369,8 @@ HBIN(H6, H6_CFG)
 #define HASH5 HASHK(H5)
 #define HASH6 HASHK(H6)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
+static_assert(kDSmem + 2048 <= 227 * 1024, "dense bin smem");
+static_assert((kDenseBits / 1024) % 32 == 0, "dense bin: top words per warp");
 #define DENSE dense_bin_kernel<1024, kDBatch, 8>
 
 static void ensure_attrs() {
