@@ -266,7 +266,7 @@ def run_aux(args):
             state["nnz"] = C.nvals
             C.free()
         ms_c = timed(step)
-        groups = ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "compact")
+        groups = ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "dense_ovf", "compact")
         kt = {k: sp.kernel_timing(k)[0] / steps for k in groups}
         sp.set_kernel_timing(False)
         clk = clocks.stop()
@@ -382,7 +382,7 @@ def main():
     log(f"[rank {rank}] step ms: {[round(x, 2) for x in step_ms]}")
     launches = sp.launch_count()
     ktimes = {k: sp.kernel_timing(k) for k in
-              ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "compact")}
+              ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "dense_ovf", "compact")}
     sp.set_kernel_timing(False)
     peak_mem = sp.memory_stats()[1]
     red_dev = "cpu" if world > 1 and dist.get_backend() == "gloo" else "cuda"

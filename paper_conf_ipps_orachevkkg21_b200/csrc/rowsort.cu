@@ -382,6 +382,16 @@ constexpr uint32_t kSlots = 16;
 template <int E>
 __device__ __forceinline__ void warp_bitonic_sort(idx_t (&x)[E]);
 
+// A hash-bin row that cannot use its table goes to a bitmap kernel: rows whose
+// span fits two small windows to list 0 (items [ovf_cnt[0] = 0, ovf_cnt[1])),
+// the others to list 1 (items [ovf_cnt[2] = nrows, ovf_cnt[3]), ovf_cnt[3]
+// starting at nrows): each pair is the bounds of one bitmap kernel launch.
+constexpr uint32_t kSmallSpan = 2u << 18;
+__device__ __forceinline__ void push_fallback(idx_t r, uint32_t span_m1, idx_t* ovf_rows, uint32_t* ovf_cnt) {
+    if (span_m1 < kSmallSpan) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+    else ovf_rows[atomicAdd(ovf_cnt + 3, 1u)] = r;
+}
+
 // Per-row work record of the hash bins (written by make_recs_kernel after
 // binning): one 40-B load gives everything the row needs.
 struct RowRec {
@@ -578,7 +588,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
         }
         PROBE(1);
         if (P.mode == kPlanWide) {
-            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            if (threadIdx.x == 0) push_fallback(r, P.rec.chi - P.rec.clo, ovf_rows, ovf_cnt);
             publish_next();
             __syncthreads();
             const RowPlan N = s_plan[(it + 1) & 1];
@@ -723,7 +733,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             fallback = s_flag != 0;
         }
         if (fallback) {
-            if (threadIdx.x == 0) ovf_rows[atomicAdd(ovf_cnt + 1, 1u)] = r;
+            if (threadIdx.x == 0) push_fallback(r, P.rec.chi - P.rec.clo, ovf_rows, ovf_cnt);
         } else {
             PROBE(5);
             // ---- multi-scan: output offset of every owned pair (one barrier) -----
@@ -861,16 +871,20 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
 }
 
 // ---- 4c. block two-level bitmap bin ------------------------------------------
-// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | bm[kDenseBits/32] | top[kDenseBits/1024]
+// dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | bm[BITS/32] | top[BITS/1024]
 // top bit t set <=> bm word t may be non-zero.  Emission walks the top level,
-// so clearing and emitting cost O(words touched + kDenseBits/1024).
-template <int THREADS, uint32_t BATCH, int FLATU>
+// so clearing and emitting cost O(words touched + BITS/1024).  Two configs:
+// 1024 threads x 1.5 Mi-bit windows, one block per SM (the dense bin: rows
+// with > 40960 products) and 256 threads x 256 Ki-bit windows, 5 blocks per
+// SM (hash-bin rows that fell back - e.g. duplicate-heavy closure rows - and
+// whose span fits two windows).
+template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS>
 __global__ void __launch_bounds__(THREADS)
 dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
                  const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
                  const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts, uint32_t* __restrict__ work) {
     constexpr int NW = THREADS / 32;
-    constexpr uint32_t kWords = kDenseBits / 32, kTop = kWords / 32;
+    constexpr uint32_t kWords = BITS / 32, kTop = kWords / 32;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const idx_t** sd_ptr = reinterpret_cast<const idx_t**>(smem_raw);
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
@@ -895,12 +909,12 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             chi = rg.y;
         }
         const uint64_t span = uint64_t(chi) - clo + 1;
-        const uint32_t nwin = uint32_t((span + kDenseBits - 1) / kDenseBits);
+        const uint32_t nwin = uint32_t((span + BITS - 1) / BITS);
         idx_t* out = scratch + soff[r];
         uint32_t written = 0;
         for (uint32_t w = 0; w < nwin; ++w) {
-            const uint64_t wlo = uint64_t(clo) + uint64_t(w) * kDenseBits;
-            const uint64_t whi = min(wlo + kDenseBits, uint64_t(chi) + 1);
+            const uint64_t wlo = uint64_t(clo) + uint64_t(w) * BITS;
+            const uint64_t whi = min(wlo + BITS, uint64_t(chi) + 1);
             block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH, false,
                                            [&](idx_t c) {
                 if (c >= wlo && c < whi) {
@@ -1371,7 +1385,11 @@ HBIN(H6, H6_CFG)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
 static_assert(kDSmem + 2048 <= 227 * 1024, "dense bin smem");
 static_assert((kDenseBits / 1024) % 32 == 0, "dense bin: top words per warp");
-#define DENSE dense_bin_kernel<1024, kDBatch, 8>
+#define DENSE dense_bin_kernel<1024, kDBatch, 8, kDenseBits>
+constexpr uint32_t kSDenseBits = 1u << 18, kSDBatch = 256;
+constexpr size_t kSDSmem = kSDBatch * kSegBytes + (kSDenseBits / 32 + kSDenseBits / 1024) * sizeof(uint32_t);
+static_assert(5 * (kSDSmem + 2048) <= 228 * 1024, "small dense bin residency");
+#define SDENSE dense_bin_kernel<256, kSDBatch, 4, kSDenseBits>
 
 static void ensure_attrs() {
     static int done_dev = -1;
@@ -1384,6 +1402,7 @@ static void ensure_attrs() {
     CUDA_CHECK(cudaFuncSetAttribute(HASH5, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H5_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(HASH6, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H6_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(DENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDSmem)));
+    CUDA_CHECK(cudaFuncSetAttribute(SDENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kSDSmem)));
     done_dev = ctx().device;
 }
 
@@ -1402,14 +1421,19 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    // meta: hist[13] binoff[14] cursor[13] work[9] ovf[2]
+    // meta: hist[13] binoff[14] cursor[13] work[9] ovf[4] work2[1]
     DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
     uint32_t* binoff = meta.p + 13;
     uint32_t* cursor = meta.p + 27;
     uint32_t* work = meta.p + 40;
-    uint32_t* ovf = meta.p + 49;  // ovf[0] = 0 (list start), ovf[1] = count
+    uint32_t* ovf = meta.p + 49;  // fallback lists: [0, ovf[1]) and [nrows, ovf[3])
+    uint32_t* work2 = meta.p + 53;
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
+    {
+        const uint32_t lst1[2] = {nrows, nrows};
+        copy_async(ovf + 2, lst1, sizeof(lst1), cudaMemcpyHostToDevice);
+    }
     const unsigned gb = (unsigned)std::min<uint64_t>(ceil_div(nrows, 256), uint64_t(nsm) * 8);
     bin_count_kernel<<<gb, 256, 0, st>>>(ub, nrows, ncols, cap.p, bin.p, counts.p, hist);
     count_launch();
@@ -1429,7 +1453,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     trace_mark("binning");
     // the scratch is matrix storage: compacted in place it becomes colidx
     DevBuf<idx_t> scratch(scratch_total, kMat);
-    DevBuf<idx_t> ovf_rows(nrows);
+    DevBuf<idx_t> ovf_rows(2 * size_t(nrows));
     DevBuf<RowRec> recs(nrows);  // indexed by bin item (only hash-bin items are written)
     make_recs_kernel<<<gb, 256, 0, st>>>(src, rows.p, binoff, ub, range, ncols, soff.p, recs.p);
     count_launch();
@@ -1458,7 +1482,11 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     LAUNCH_HASH(HASH0, H0, BIN_H0, 8)
 #undef LAUNCH_HASH
     // rows whose hash probes ran long: bitmap path
-    DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work + 6);
+    t = ktime_begin("dense_ovf", st);
+    SDENSE<<<nsm * 5, 256, kSDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work2);
+    DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf + 2, range, ncols, scratch.p, soff.p, counts.p, work + 6);
+    ktime_end(t);
+    count_launch();
     count_launch(9);
     check_launch("block bins");
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
