@@ -9,7 +9,10 @@ for so in paper_conf_ipps_orachevkkg21_b200/variants/libspbla_*.so; do
     python -c "
 import json
 d=json.load(open('$O/$name.$wl.json'))
-print('$name', '$wl', round(d['ms_per_step'],2),'ms', {k: round(v,2) for k,v in d['roofline']['kernel_ms_per_step'].items() if k[0] in 'Hw'})
+if 'roofline' in d:
+    print('$name', '$wl', round(d['ms_per_step'],2),'ms', {k: round(v,2) for k,v in d['roofline']['kernel_ms_per_step'].items() if k[0] in 'Hwd'})
+else:
+    print('$name', '$wl', round(d['value'],2),'ms', {k: round(v,2) for k,v in d['kernel_ms_per_step'].items() if k[0] in 'Hwd'})
 " 2>&1 | tee -a $O/summary.txt || tail -3 $O/$name.$wl.err
   done
 done
