@@ -175,6 +175,33 @@ def test_mxm_heavy_rows_multiwindow(sp):
     assert_same(sp.mxm(A, B), oracle.mxm(OA, OB), "heavy")
 
 
+@pytest.mark.parametrize("ncols,label", [(1 << 18, "narrow span: small bitmap fallback"),
+                                         (1 << 22, "wide span: large bitmap fallback")])
+def test_mxm_duplicate_heavy_fallback(sp, ncols, label):
+    """Hash-bin rows whose products are ~50 copies of ~50 columns (closure-like):
+    buckets overflow with duplicates, the rows fall back to a bitmap kernel
+    chosen by span (2^18 columns: the 256-thread small-window kernel; 2^22: the
+    1.5 Mi-window one).  Mixed with ordinary rows in the same launch."""
+    rng = np.random.default_rng(77)
+    hub_cols = np.sort(rng.choice(ncols, 50, replace=False)).astype(np.uint32)
+    nb_hub = 64
+    # B: 64 hub rows sharing the same 50 columns, 400 ordinary rows of 8 random columns
+    rb = np.concatenate([np.repeat(np.arange(nb_hub), 50), np.repeat(np.arange(nb_hub, nb_hub + 400), 8)])
+    cb = np.concatenate([np.tile(hub_cols, nb_hub), rng.integers(0, ncols, 400 * 8)])
+    # A: rows 0..299 take 30..60 hub rows (1500..3000 products, 50 distinct);
+    # rows 300..599 take 100 ordinary rows (800 products, mostly distinct)
+    ra, ca = [], []
+    for i in range(300):
+        k = rng.choice(nb_hub, rng.integers(30, 61), replace=False)
+        ra += [i] * len(k); ca += list(k)
+    for i in range(300, 600):
+        k = rng.choice(np.arange(nb_hub, nb_hub + 400), 100, replace=False)
+        ra += [i] * len(k); ca += list(k)
+    A, OA = both_from_pairs(sp, 600, nb_hub + 400, np.array(ra, np.uint32), np.array(ca, np.uint32))
+    B, OB = both_from_pairs(sp, nb_hub + 400, ncols, rb.astype(np.uint32), cb.astype(np.uint32))
+    assert_same(sp.mxm(A, B), oracle.mxm(OA, OB), label)
+
+
 # ------------------------------------------------------------------ EWiseAdd
 
 @pytest.mark.parametrize("seed", range(3))
