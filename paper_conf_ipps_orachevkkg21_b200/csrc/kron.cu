@@ -14,35 +14,37 @@ namespace spbla {
 
 namespace {
 
-__global__ void kron_rowptr_kernel(CsrView A, CsrView B, uint64_t nnzB, off_t64* __restrict__ rp) {
+// Eight lanes per K row (four rows per warp in flight: rows average tens of
+// items, so a warp per row would idle most lanes behind its dependent
+// row-offset loads).  The row offset comes from the closed form (lane 0 of
+// the group also stores it, so one launch writes both arrays); lane l walks
+// items e = l, l+8, ... keeping (e / lb, e % lb) incrementally.
+constexpr unsigned kKG = 8;
+__global__ void kron_kernel(CsrView A, CsrView B, uint64_t nnzB, off_t64* __restrict__ rp, idx_t* __restrict__ out) {
     const uint64_t n = uint64_t(A.nrows) * B.nrows;
-    for (uint64_t r = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; r <= n;
-         r += uint64_t(gridDim.x) * blockDim.x) {
-        if (r == n) {
-            rp[r] = A.rowptr[A.nrows] * nnzB;
-            continue;
-        }
-        const idx_t ia = idx_t(r / B.nrows), ib = idx_t(r - uint64_t(ia) * B.nrows);
-        const uint64_t la = A.rowptr[ia + 1] - A.rowptr[ia];
-        rp[r] = A.rowptr[ia] * nnzB + la * B.rowptr[ib];
-    }
-}
-
-// One warp per K row; the row's la*lb items are spread over the 32 lanes.
-__global__ void kron_cols_kernel(CsrView A, CsrView B, const off_t64* __restrict__ rp,
-                                 idx_t* __restrict__ out) {
-    const uint64_t n = uint64_t(A.nrows) * B.nrows;
-    const unsigned lane = lane_id();
-    const uint64_t nw = uint64_t(gridDim.x) * (blockDim.x >> 5);
-    for (uint64_t r = (blockIdx.x * uint64_t(blockDim.x) + threadIdx.x) >> 5; r < n; r += nw) {
+    const unsigned gl = threadIdx.x & (kKG - 1);
+    const uint64_t ng = uint64_t(gridDim.x) * (blockDim.x / kKG);
+    const uint64_t r0 = (blockIdx.x * uint64_t(blockDim.x) + threadIdx.x) / kKG;
+    if (r0 == 0 && gl == 0) rp[n] = A.rowptr[A.nrows] * nnzB;
+    for (uint64_t r = r0; r < n; r += ng) {
         const idx_t ia = idx_t(r / B.nrows), ib = idx_t(r - uint64_t(ia) * B.nrows);
         const off_t64 sa = A.rowptr[ia], sb = B.rowptr[ib];
-        const uint32_t lb = uint32_t(B.rowptr[ib + 1] - sb);
-        const uint64_t cnt = uint64_t(A.rowptr[ia + 1] - sa) * lb;
-        idx_t* o = out + rp[r];
-        for (uint64_t e = lane; e < cnt; e += 32) {
-            const uint64_t a = e / lb, b = e - a * lb;
-            o[e] = A.colidx[sa + a] * B.ncols + B.colidx[sb + b];
+        const uint32_t la = uint32_t(A.rowptr[ia + 1] - sa), lb = uint32_t(B.rowptr[ib + 1] - sb);
+        const uint64_t base = sa * nnzB + uint64_t(la) * sb;
+        if (gl == 0) rp[r] = base;
+        const uint64_t cnt = uint64_t(la) * lb;
+        if (cnt == 0) continue;
+        idx_t* o = out + base;
+        const uint32_t da = kKG / lb, db = kKG % lb;
+        uint32_t ai = gl / lb, bi = gl % lb;
+        for (uint64_t e = gl; e < cnt; e += kKG) {
+            o[e] = A.colidx[sa + ai] * B.ncols + B.colidx[sb + bi];
+            ai += da;
+            bi += db;
+            if (bi >= lb) {
+                bi -= lb;
+                ++ai;
+            }
         }
     }
 }
@@ -59,18 +61,12 @@ void kronecker(Matrix* K, const Matrix* A, const Matrix* B) {
     DevBuf<off_t64> rp(m + 1, kMat);
     DevBuf<idx_t> ci(nnz, kMat);
     const int nsm = ctx().num_sms;
-    unsigned g1 = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(m + 1, 256), uint64_t(nsm) * 16));
     const int t = ktime_begin("kron", ctx().stream);
-    kron_rowptr_kernel<<<g1, 256, 0, ctx().stream>>>(view(A), view(B), B->nnz, rp.p);
-    count_launch();
-    check_launch("kron_rowptr_kernel");
-    if (nnz) {
-        unsigned g2 = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(m * 32, 256), uint64_t(nsm) * 32));
-        kron_cols_kernel<<<g2, 256, 0, ctx().stream>>>(view(A), view(B), rp.p, ci.p);
-        count_launch();
-        check_launch("kron_cols_kernel");
-    }
+    const unsigned g = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(m * kKG, 256), uint64_t(nsm) * 8));
+    kron_kernel<<<g, 256, 0, ctx().stream>>>(view(A), view(B), B->nnz, rp.p, ci.p);
     ktime_end(t);
+    count_launch();
+    check_launch("kron_kernel");
     size_t rc = rp.n, cc = ci.n;
     matrix_replace(K, rp.detach(), rc, ci.detach(), cc, nnz);
 }
