@@ -69,7 +69,7 @@ for rep in sorted(glob.glob(os.path.join(CK, "top_*.ncu-rep"))):
     out.append("")
 
 # 3. bench lines
-for f in ("bench.json", "bench_ref.json", "bench_2rank_gloo.json"):
+for f in ("bench.json", "bench_ref.json", "bench_2rank_gloo.json", "bench_ewise_kron.json", "bench_closure18.json"):
     p = os.path.join(CK, f)
     if os.path.exists(p) and os.path.getsize(p):
         out.append(f"## {f}\n\n```json\n{open(p).read().strip()}\n```\n")
@@ -78,7 +78,7 @@ if traffic:
     tp = os.path.join(P, "ncu_traffic.json")
     tj = json.load(open(tp)) if os.path.exists(tp) else {}
     for grp, (byt, kname) in traffic.items():
-        tj.setdefault("rmat22_ef32", {})[grp] = byt
+        tj.setdefault("ewise_kron" if grp.startswith("ewise") else "rmat22_ef32", {})[grp] = byt
         tj.setdefault("_source", {})[grp] = f"profiles/{tag}_summary.md: {kname[:80]}"
     json.dump(tj, open(tp, "w"), indent=1)
 print(open(os.path.join(P, f"{tag}_summary.md")).read()[:3000])
