@@ -455,7 +455,8 @@ __host__ __device__ constexpr uint32_t first_entries(uint64_t maxub) { return ui
 //               ovl[OVCAP] | pool[OVCAP] u16 | obl[OBCAP] | obcnt[OBCAP] | poff[MAXB/2]
 // (the per-warp overflow buffers wbuf[THREADS] alias the segment descriptors,
 // which are dead once the products are inserted: BATCH * 3 >= THREADS)
-template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU, bool DEDUP_B>
+template <int THREADS, uint32_t MAXB, uint32_t OVCAP, uint32_t OBCAP, uint32_t BATCH, int MINB, int FLATU, bool DEDUP_B,
+          int KIND>
 __global__ void __launch_bounds__(THREADS, MINB)
 hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* __restrict__ bounds,
                 idx_t* __restrict__ scratch, uint32_t* __restrict__ counts,
@@ -489,7 +490,8 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
     const uint32_t lo_i = bounds[0], hi_i = bounds[1];
-    const bool pre = src.kind == 0;  // descriptor mode: first batches are prefetched
+    src.kind = KIND;  // compile-time segment source: the helpers' kind branches fold away
+    const bool pre = KIND == 0;  // descriptor mode: first batches are prefetched
     RowPlan end_plan;
     end_plan.mode = kPlanEnd;
     // descriptor prefetch of a row's first batch: issue (loads in flight) ...
@@ -1374,14 +1376,14 @@ HBIN(H5, H5_CFG)
 #define H6_CFG 1024, kH6, 192, 96, 384, 1, 4, true
 #endif
 HBIN(H6, H6_CFG)
-#define HASHK(N) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U, N##_DB>
-#define HASH0 HASHK(H0)
-#define HASH1 HASHK(H1)
-#define HASH2 HASHK(H2)
-#define HASH3 HASHK(H3)
-#define HASH4 HASHK(H4)
-#define HASH5 HASHK(H5)
-#define HASH6 HASHK(H6)
+#define HASHK(N, KIND) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U, N##_DB, KIND>
+#define HASH0(KIND) HASHK(H0, KIND)
+#define HASH1(KIND) HASHK(H1, KIND)
+#define HASH2(KIND) HASHK(H2, KIND)
+#define HASH3(KIND) HASHK(H3, KIND)
+#define HASH4(KIND) HASHK(H4, KIND)
+#define HASH5(KIND) HASHK(H5, KIND)
+#define HASH6(KIND) HASHK(H6, KIND)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
 static_assert(kDSmem + 2048 <= 227 * 1024, "dense bin smem");
 static_assert((kDenseBits / 1024) % 32 == 0, "dense bin: top words per warp");
@@ -1394,13 +1396,20 @@ static_assert(5 * (kSDSmem + 2048) <= 228 * 1024, "small dense bin residency");
 static void ensure_attrs() {
     static int done_dev = -1;
     if (done_dev == ctx().device) return;
-    CUDA_CHECK(cudaFuncSetAttribute(HASH0, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H0_SMEM)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH1, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H1_SMEM)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH2, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H2_SMEM)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH3, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H3_SMEM)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH4, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H4_SMEM)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH5, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H5_SMEM)));
-    CUDA_CHECK(cudaFuncSetAttribute(HASH6, cudaFuncAttributeMaxDynamicSharedMemorySize, int(H6_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH0(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H0_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH0(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H0_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH1(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H1_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH1(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H1_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH2(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H2_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH2(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H2_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH3(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H3_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH3(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H3_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH4(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H4_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH4(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H4_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH5(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H5_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH5(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H5_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH6(0), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H6_SMEM)));
+    CUDA_CHECK(cudaFuncSetAttribute(HASH6(1), cudaFuncAttributeMaxDynamicSharedMemorySize, int(H6_SMEM)));
     CUDA_CHECK(cudaFuncSetAttribute(DENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kDSmem)));
     CUDA_CHECK(cudaFuncSetAttribute(SDENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kSDSmem)));
     done_dev = ctx().device;
@@ -1468,10 +1477,14 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DENSE<<<nsm, 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols, scratch.p, soff.p,
                                      counts.p, work);
     ktime_end(t);
-#define LAUNCH_HASH(K, NAME, BIN, W)                                                                  \
-    t = ktime_begin(#NAME, st);                                                                         \
-    K<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p, counts.p,  \
-                                                         work + W, ovf_rows.p, ovf);                    \
+#define LAUNCH_HASH(K, NAME, BIN, W)                                                                   \
+    t = ktime_begin(#NAME, st);                                                                          \
+    if (src.kind == 0)                                                                                   \
+        K(0)<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p,    \
+                                                                counts.p, work + W, ovf_rows.p, ovf);   \
+    else                                                                                                 \
+        K(1)<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p,    \
+                                                                counts.p, work + W, ovf_rows.p, ovf);   \
     ktime_end(t);
     LAUNCH_HASH(HASH6, H6, BIN_H6, 7)
     LAUNCH_HASH(HASH5, H5, BIN_H5, 1)
