@@ -17,10 +17,18 @@ namespace {
 
 constexpr int kGroup = 8;
 
-// Column span of every B row: bspan[k] = (B[k][0], B[k][last]) (rows are
-// sorted), (0xFFFFFFFF, 0) for an empty row.  8 B per row: the upper-bound
-// pass then reads one L2-resident word per A entry instead of two scattered
-// colidx sectors.
+// Per-B-row info, one 16-B record: binfo[k] = (start, length, first column,
+// last column) (rows are sorted; (0xFFFFFFFF, 0) as span of an empty row).
+// The upper-bound pass then reads one aligned sector per A entry instead of
+// the row-offset pair and two scattered colidx sectors.  32-bit starts need
+// nnz(B) < 2^32; larger B keeps 64-bit offsets (binfo = null).
+__global__ void row_info_kernel(CsrView B, uint4* __restrict__ binfo) {
+    for (size_t k = blockIdx.x * size_t(blockDim.x) + threadIdx.x; k < B.nrows; k += size_t(gridDim.x) * blockDim.x) {
+        const off_t64 x = B.rowptr[k], y = B.rowptr[k + 1];
+        binfo[k] = y > x ? make_uint4(uint32_t(x), uint32_t(y - x), B.colidx[x], B.colidx[y - 1])
+                         : make_uint4(uint32_t(x), 0u, 0xFFFFFFFFu, 0u);
+    }
+}
 __global__ void row_span_kernel(CsrView B, uint2* __restrict__ bspan) {
     for (size_t k = blockIdx.x * size_t(blockDim.x) + threadIdx.x; k < B.nrows; k += size_t(gridDim.x) * blockDim.x) {
         const off_t64 x = B.rowptr[k], y = B.rowptr[k + 1];
@@ -28,8 +36,10 @@ __global__ void row_span_kernel(CsrView B, uint2* __restrict__ bspan) {
     }
 }
 
+template <bool INFO>
 __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
-                              const uint2* __restrict__ bspan, const off_t64* __restrict__ crp,
+                              const uint2* __restrict__ bspan, const uint4* __restrict__ binfo,
+                              const off_t64* __restrict__ crp,
                               const idx_t* __restrict__ cci, uint64_t* __restrict__ ub, uint2* __restrict__ range,
                               uint4* __restrict__ desc, uint32_t* __restrict__ nseg) {
     const unsigned lane = threadIdx.x & 31, g = lane & (kGroup - 1);
@@ -72,12 +82,20 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
             uint64_t ptr = 0;
             if (valid && p < e) {
                 const idx_t k = A.colidx[p];
-                const off_t64 x = brp[k], y = brp[k + 1];
-                const uint2 sp = bspan[k];  // (0xFFFFFFFF, 0) when empty: neutral
-                len = uint32_t(y - x);
-                ptr = reinterpret_cast<uint64_t>(bci + x);
-                lo = min(lo, sp.x);
-                hi = max(hi, sp.y);
+                if (INFO) {
+                    const uint4 bi = binfo[k];  // span (0xFFFFFFFF, 0) when empty: neutral
+                    len = bi.y;
+                    ptr = reinterpret_cast<uint64_t>(bci + bi.x);
+                    lo = min(lo, bi.z);
+                    hi = max(hi, bi.w);
+                } else {
+                    const off_t64 x = brp[k], y = brp[k + 1];
+                    const uint2 sp = bspan[k];  // (0xFFFFFFFF, 0) when empty: neutral
+                    len = uint32_t(y - x);
+                    ptr = reinterpret_cast<uint64_t>(bci + x);
+                    lo = min(lo, sp.x);
+                    hi = max(hi, sp.y);
+                }
             }
             s += len;
             // compacted position and inclusive length prefix inside the group
@@ -130,15 +148,24 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     const unsigned grid = (unsigned)std::min<uint64_t>(ceil_div(uint64_t(m) * kGroup, 256),
                                                        uint64_t(ctx().num_sms) * 16);
     const off_t64* crp = accumulate ? C->rowptr : nullptr;
-    DevBuf<uint2> bspan(B->nrows);
+    const bool info = B->nnz < (uint64_t(1) << 32);
+    DevBuf<uint4> binfo(info ? B->nrows : 0);
+    DevBuf<uint2> bspan(info ? 0 : B->nrows);
     int tk = ktime_begin("mxm_ub", ctx().stream);
     if (B->nrows) {
         const unsigned gs = (unsigned)std::min<uint64_t>(ceil_div(B->nrows, 256), uint64_t(ctx().num_sms) * 16);
-        row_span_kernel<<<gs, 256, 0, ctx().stream>>>(view(B), bspan.p);
+        if (info) row_info_kernel<<<gs, 256, 0, ctx().stream>>>(view(B), binfo.p);
+        else row_span_kernel<<<gs, 256, 0, ctx().stream>>>(view(B), bspan.p);
         count_launch();
     }
-    mxm_ub_kernel<<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, bspan.p, crp,
-                                                  accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p, nseg.p);
+    if (info)
+        mxm_ub_kernel<true><<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, nullptr, binfo.p, crp,
+                                                            accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p,
+                                                            nseg.p);
+    else
+        mxm_ub_kernel<false><<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, bspan.p, nullptr, crp,
+                                                             accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p,
+                                                             nseg.p);
     ktime_end(tk);
     count_launch();
     check_launch("mxm_ub_kernel");

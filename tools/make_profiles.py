@@ -21,7 +21,7 @@ for r in rows[hi + 1:]:
     m = re.search(r'(\w+_kernel)(<[^>]*>)?', name)
     seq.append(((m.group(1) + (m.group(2) or '')) if m else name[:60], v, 'spbla' in name))
 # last step = from the last row_span_kernel (first launch of an MxM) to the end
-last = max(i for i, s in enumerate(seq) if s[0].startswith('row_span_kernel'))
+last = max(i for i, s in enumerate(seq) if s[0].startswith(('row_span_kernel', 'row_info_kernel')))
 step = [s for s in seq[last:] if s[2]]
 tot = sum(v for _, v, _ in step)
 out.append(f"# {tag}: ncu launch list of one bench.py step (configs[4], rmat22_ef32 A.A)\n")
