@@ -402,6 +402,11 @@ struct RowRec {
 // A row's plan, computed once by thread 0 (one row ahead) and read by all
 // threads from shared memory: mode, bucket count, width and exact reciprocal.
 enum : uint32_t { kPlanHash = 0, kPlanBitmap = 1, kPlanWide = 2, kPlanEnd = 3 };
+// mean bucket load: nb = ub / kLoadDiv buckets of 16 slots
+#ifndef SPBLA_LOAD_DIV
+#define SPBLA_LOAD_DIV 8
+#endif
+constexpr uint32_t kLoadDiv = SPBLA_LOAD_DIV;
 struct RowPlan {
     RowRec rec;
     uint32_t mode, nb, W, l, M, nw;
@@ -415,7 +420,7 @@ __device__ __forceinline__ RowPlan make_plan(const RowRec& x) {
     // table goes to the bitmap bin.  nb is even (buckets are sorted in pairs).
     const uint64_t nbw = (span + 65534) / 65535;
     const uint32_t nb =
-        (uint32_t(min(max(max(uint64_t((x.u + 7) / 8), nbw), uint64_t(1)), uint64_t(MAXB))) + 1) & ~1u;
+        (uint32_t(min(max(max(uint64_t((x.u + kLoadDiv - 1) / kLoadDiv), nbw), uint64_t(1)), uint64_t(MAXB))) + 1) & ~1u;
     const uint64_t words = (span + 31) >> 5;
     P.nb = nb;
     P.nw = uint32_t(min(words, uint64_t(0xFFFFFFFFu)));
