@@ -75,9 +75,13 @@ def load_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    """nvidia-smi clocks / throttle reasons sampled during the timed region.
 
-    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+    The sampler is started before the warm-up (nvidia-smi's start-up must not
+    land in the first timed step) and only samples whose timestamps fall in
+    [window()] are kept (all samples if the timestamps cannot be parsed)."""
+
+    FIELDS = ("timestamp,clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
 
@@ -92,7 +96,13 @@ class ClockSampler:
         except Exception:
             self.proc = None
 
+    t0 = t1 = None
+
+    def window(self, t0, t1):
+        self.t0, self.t1 = t0, t1
+
     def stop(self):
+        import datetime
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         self.proc.terminate()
@@ -101,18 +111,27 @@ class ClockSampler:
         except Exception:
             self.proc.kill()
         self.out.seek(0)
-        sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        rows = []
         for line in self.out.read().splitlines():
             f = [x.strip() for x in line.split(",")]
-            if len(f) < 7:
+            if len(f) < 8:
                 continue
             try:
-                sm.append(float(f[0]))
-                mx.append(float(f[1]))
+                ts = datetime.datetime.strptime(f[0], "%Y/%m/%d %H:%M:%S.%f").timestamp()
+            except ValueError:
+                ts = None
+            try:
+                rows.append((ts, float(f[1]), float(f[2]), f[4:8]))
             except ValueError:
                 continue
-            for nm, v in zip(names, f[3:7]):
+        inwin = [x for x in rows if x[0] is not None and self.t0 is not None and self.t0 - 0.25 <= x[0] <= self.t1 + 0.25]
+        use = inwin if inwin else rows
+        sm = [x[1] for x in use]
+        mx = [x[2] for x in use]
+        reasons = set()
+        for x in use:
+            for nm, v in zip(names, x[3]):
                 if v.lower() == "active":
                     reasons.add(nm)
         self.out.close()
@@ -197,7 +216,9 @@ def run_aux(args):
     launches = []
 
     def timed(fn):
-        for _ in range(warmup):
+        for i in range(warmup):
+            if i == warmup - 1:
+                sp.set_kernel_timing(True)
             fn()
         torch.cuda.synchronize()
         sp.set_kernel_timing(True)
@@ -351,22 +372,10 @@ def main():
         return C
 
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device="cuda")
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    nnzC_local = C.nvals
-
-    # ---- timed region ------------------------------------------------------------
-    sp.reset_peak_memory()
-    sp.reset_launch_count()
-    if not os.environ.get("BENCH_NO_KTIME"):
-        sp.set_kernel_timing(True)
-    clocks = ClockSampler(local)
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    step_ms = []
-    for _ in range(args.steps):
+    clocks = ClockSampler(local)  # started before the warm-up: its start-up stays out of the timed steps
+    ktime = not os.environ.get("BENCH_NO_KTIME")
+    def timed_step():
+        # the same body for the warm-up and the timed steps (L2 flush, events)
         flush.zero_()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
@@ -374,10 +383,29 @@ def main():
         step()
         e1.record(stream)
         e1.synchronize()
-        step_ms.append(e0.elapsed_time(e1))
+        return e0.elapsed_time(e1)
+
+    for i in range(args.warmup):
+        if ktime and i == args.warmup - 1:
+            sp.set_kernel_timing(True)  # event pool warmed up in the last warm-up step
+        timed_step()
+    torch.cuda.synchronize()
+    nnzC_local = C.nvals
+
+    # ---- timed region ------------------------------------------------------------
+    sp.reset_peak_memory()
+    sp.reset_launch_count()
+    if ktime:
+        sp.set_kernel_timing(True)  # (clears the warm-up records)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_begin = time.time()
+    step_ms = [timed_step() for _ in range(args.steps)]
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
+    clocks.window(t_begin, time.time())
     clk = clocks.stop()
     log(f"[rank {rank}] step ms: {[round(x, 2) for x in step_ms]}")
     launches = sp.launch_count()

@@ -1347,7 +1347,7 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
     constexpr uint32_t NAME##_B = uint32_t(UB / 8), NAME##_OVCAP = OVCAP, NAME##_OBCAP = OBCAP,     \
                        NAME##_BATCH = BATCH;                                                       \
     constexpr size_t NAME##_SMEM = hash_smem(T, BATCH, uint32_t(UB / 8), OVCAP, OBCAP);            \
-    static_assert(PERSM * (NAME##_SMEM + 1024 + 1200) <= 228 * 1024, #NAME " residency");         \
+    static_assert(PERSM * (NAME##_SMEM + 1024 + 512) <= 228 * 1024, #NAME " residency");         \
     static_assert(PERSM * T <= 2048, #NAME " threads");
 // <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread,
 //  dedup in pass B (else re-sort in pass A)>
@@ -1370,7 +1370,7 @@ HBIN(H2, H2_CFG)
 #endif
 HBIN(H3, H3_CFG)
 #ifndef H4_CFG  // (overridable for tools/sweep.sh)
-#define H4_CFG 256, kH4, 64, 32, 256, 4, 6, false
+#define H4_CFG 256, kH4, 64, 32, 256, 5, 6, false
 #endif
 HBIN(H4, H4_CFG)
 #ifndef H5_CFG  // (overridable for tools/sweep.sh)
