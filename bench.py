@@ -214,6 +214,7 @@ def run_aux(args):
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device="cuda")
     steps, warmup = args.steps, max(args.warmup, 3)
     launches = []
+    step_lists = []
 
     def timed(fn):
         for i in range(warmup):
@@ -234,7 +235,11 @@ def run_aux(args):
             e1.synchronize()
             ms.append(e0.elapsed_time(e1))
         launches.append(sp.launch_count())
-        return sum(ms) / len(ms)
+        log(f"[aux] step ms: {[round(x, 2) for x in ms]}")
+        step_lists.append([round(x, 3) for x in ms])
+        # median: these host-launch-bound ops see occasional 10-200 ms host
+        # stalls in pool allocations; the full list is reported
+        return statistics.median(ms)
 
     clocks = ClockSampler(0)
     if args.workload == "ewise_kron":
@@ -299,6 +304,8 @@ def run_aux(args):
                            "l2": "256 MB write between timed steps"},
                 "ms_per_iteration": ms_c / state["it"], "kernel_ms_per_step": kt, "clocks": clk}
     line["gpu_launches"] = sum(launches)
+    line["step_ms"] = step_lists
+    line["value_is"] = "median of the timed steps (each step list in step_ms)"
     print(json.dumps(line), flush=True)
 
 
