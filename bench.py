@@ -15,7 +15,6 @@ import argparse
 import json
 import os
 import statistics
-import subprocess
 import sys
 import time
 
@@ -75,68 +74,67 @@ def load_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region.
+    """SM clocks and clock-event (throttle) reasons sampled during the timed
+    region, in-process through NVML (a background thread, 100 ms period):
+    spawning nvidia-smi in a loop stalls CUDA calls of the measured process
+    for tens to hundreds of ms.  Started before the warm-up; only samples in
+    window() are kept (all samples if the window is not set)."""
 
-    The sampler is started before the warm-up (nvidia-smi's start-up must not
-    land in the first timed step) and only samples whose timestamps fall in
-    [window()] are kept (all samples if the timestamps cannot be parsed)."""
-
-    FIELDS = ("timestamp,clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-              "clocks_event_reasons.sw_power_cap")
-
-    def __init__(self, gpu_index):
-        self.proc = None
-        self.out = None
-        try:
-            self.out = open(f"/tmp/clocks_{os.getpid()}.csv", "w+")
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(gpu_index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "200"], stdout=self.out, stderr=subprocess.DEVNULL)
-        except Exception:
-            self.proc = None
-
+    NAMES = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+             "hw_power_brake_slowdown": 0x80, "sw_power_cap": 0x4}
     t0 = t1 = None
+
+    def __init__(self, gpu_index, period=0.1):
+        import threading
+        self.samples = []
+        self.stop_ev = threading.Event()
+        self.thread = None
+        if os.environ.get("BENCH_NO_CLOCKS"):
+            return
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nvml = pynvml
+            # NVML indexes physical GPUs; map through CUDA_VISIBLE_DEVICES
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            idx = int(vis.split(",")[gpu_index]) if vis and vis.split(",")[gpu_index].isdigit() else gpu_index
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            return
+
+        def run():
+            while not self.stop_ev.is_set():
+                try:
+                    mhz = self.nvml.nvmlDeviceGetClockInfo(self.h, self.nvml.NVML_CLOCK_SM)
+                    rs = self.nvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                    self.samples.append((time.time(), mhz, rs))
+                except Exception:
+                    pass
+                self.stop_ev.wait(period)
+        self.thread = threading.Thread(target=run, daemon=True)
+        self.thread.start()
 
     def window(self, t0, t1):
         self.t0, self.t1 = t0, t1
 
     def stop(self):
-        import datetime
-        if self.proc is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except Exception:
-            self.proc.kill()
-        self.out.seek(0)
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        rows = []
-        for line in self.out.read().splitlines():
-            f = [x.strip() for x in line.split(",")]
-            if len(f) < 8:
-                continue
-            try:
-                ts = datetime.datetime.strptime(f[0], "%Y/%m/%d %H:%M:%S.%f").timestamp()
-            except ValueError:
-                ts = None
-            try:
-                rows.append((ts, float(f[1]), float(f[2]), f[4:8]))
-            except ValueError:
-                continue
-        inwin = [x for x in rows if x[0] is not None and self.t0 is not None and self.t0 - 0.25 <= x[0] <= self.t1 + 0.25]
-        use = inwin if inwin else rows
-        sm = [x[1] for x in use]
-        mx = [x[2] for x in use]
+        if self.thread is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["clock sampling unavailable"]}
+        self.stop_ev.set()
+        self.thread.join(timeout=2)
+        use = self.samples
+        if self.t0 is not None:
+            win = [x for x in self.samples if self.t0 - 0.15 <= x[0] <= self.t1 + 0.15]
+            use = win or self.samples
         reasons = set()
-        for x in use:
-            for nm, v in zip(names, x[3]):
-                if v.lower() == "active":
+        for _, _, rs in use:
+            for nm, bit in self.NAMES.items():
+                if rs & bit:
                     reasons.add(nm)
-        self.out.close()
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        sm = [x[1] for x in use]
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(reasons), "samples": len(sm), "source": "NVML in-process, 100 ms"}
 
 
 # ---------------------------------------------------------------------------
