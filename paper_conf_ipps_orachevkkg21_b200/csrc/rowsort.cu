@@ -1358,15 +1358,15 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
 #endif
 HBIN(H0, H0_CFG)
 #ifndef H1_CFG  // (overridable for tools/sweep.sh)
-#define H1_CFG 32, kH1, 32, 16, 128, 24, 4, false
+#define H1_CFG 32, kH1, 32, 16, 32, 24, 4, false
 #endif
 HBIN(H1, H1_CFG)
 #ifndef H2_CFG  // (overridable for tools/sweep.sh)
-#define H2_CFG 64, kH2, 32, 16, 128, 16, 4, false
+#define H2_CFG 64, kH2, 32, 16, 64, 16, 4, false
 #endif
 HBIN(H2, H2_CFG)
 #ifndef H3_CFG  // (overridable for tools/sweep.sh)
-#define H3_CFG 128, kH3, 64, 32, 256, 8, 6, false
+#define H3_CFG 128, kH3, 64, 32, 128, 8, 6, false
 #endif
 HBIN(H3, H3_CFG)
 #ifndef H4_CFG  // (overridable for tools/sweep.sh)
