@@ -146,7 +146,10 @@ struct SegSource {
 // in `out` (nrows x ncols).  dedup=false promises rows are duplicate-free.
 // range (nullable): per-row [min col, max col] of the row's segments, needed
 // (and computed by MxM) for rows with ub > kRangeMinUb; null means [0, ncols).
-constexpr uint64_t kRangeMinUb = 256;
+#ifndef SPBLA_WARP_MAX
+#define SPBLA_WARP_MAX 256
+#endif
+constexpr uint64_t kRangeMinUb = SPBLA_WARP_MAX;
 void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, const uint2* range,
                 Matrix* out);
 

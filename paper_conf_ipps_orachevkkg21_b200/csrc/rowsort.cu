@@ -77,9 +77,9 @@ constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
 __device__ __forceinline__ int bin_of(uint64_t ub) {
     if (ub == 0) return BIN_EMPTY;
-    if (ub <= 32) return BIN_W1;
-    if (ub <= 64) return BIN_W2;
-    if (ub <= 128) return BIN_W4;
+    if (ub <= 32 && 32 <= kWarpMaxUb) return BIN_W1;
+    if (ub <= 64 && 64 <= kWarpMaxUb) return BIN_W2;
+    if (ub <= 128 && 128 <= kWarpMaxUb) return BIN_W4;
     if (ub <= kWarpMaxUb) return BIN_W8;
     if (ub <= kH0) return BIN_H0;
     if (ub <= kH1) return BIN_H1;
