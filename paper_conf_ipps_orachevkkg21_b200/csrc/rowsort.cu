@@ -197,12 +197,15 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
 // inside the run (segments average tens of products, so a run rarely
 // crosses more than one boundary); the U loads are issued before any
 // insert.  A warp covers 32*U consecutive products, i.e. a few sectors of
-// each B row.  Ends with a barrier.
+// each B row.  Ends with a barrier.  abort (optional): a shared flag; once it
+// is set every thread skips the rest of its products (the caller discards
+// the row).
 // prestaged: the first batch is already staged (and visible to all threads).
 template <int THREADS, int U, typename F>
 __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint64_t sbase, uint32_t nseg,
                                                const idx_t** sd_ptr, uint32_t* sd_end, uint32_t* sd_first,
-                                               uint32_t batch, bool prestaged, F&& f) {
+                                               uint32_t batch, bool prestaged, F&& f,
+                                               const volatile uint32_t* abort = nullptr) {
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
         const uint32_t ns = min(batch, nseg - s0);
         const uint32_t total = (s0 == 0 && prestaged)
@@ -212,6 +215,9 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
         for (uint32_t q0 = threadIdx.x * U; q0 < total; q0 += THREADS * U) {
+            // a row already bound for the fallback stops gathering (per
+            // thread: no barrier inside this loop)
+            if (abort && *abort) break;
             uint32_t k;
             if (s.kind == 1) {
                 k = 0;
@@ -490,7 +496,14 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     static_assert(BATCH * 3 >= THREADS && OVCAP % 2 == 0 && MAXB % 2 == 0 && MP % 32 == 0, "hash bin layout");
     __shared__ uint32_t s_w[33];
     __shared__ uint32_t s_wt[KP][NW];
-    __shared__ uint32_t s_flag, s_novf, s_nob, s_pool;
+    // s_flag / s_novf are written (and s_flag read) during the gather, which
+    // starts without a barrier: they alternate by row parity, and row i
+    // clears row i+1's pair (row i-1's last reads precede the barrier that
+    // ended row i-1)
+    __shared__ uint32_t s_flag2[2], s_novf2[2], s_nob, s_pool;
+    // early stop of the gather once the row is bound for the fallback: the
+    // small bins, where duplicate-heavy closure rows overflow
+    constexpr bool kEarlyStop = THREADS <= 128;
     __shared__ RowPlan s_plan[2];
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
@@ -526,6 +539,10 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     for (uint32_t i = threadIdx.x; i < TABW; i += THREADS) tabw[i] = 0xFFFFFFFFu;
 #pragma unroll 1
     for (uint32_t i = threadIdx.x; i < MAXB; i += THREADS) bcnt[i] = 0u;
+    if (threadIdx.x == 0) {
+        s_flag2[0] = s_flag2[1] = 0;
+        s_novf2[0] = s_novf2[1] = 0;
+    }
     // prologue: claim rows 0 and 1, plan row 0, stage its first batch
     // the pipeline thread is the last one: it has the least pass-A work
     constexpr unsigned PT = THREADS - 1;
@@ -554,9 +571,13 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             have_nx = nxt1 < hi_i;
             if (have_nx) nx = recs[nxt1];
         }
+        // (single-buffered in the bins without the early stop, as before)
+        const uint32_t fcur = kEarlyStop ? (it & 1) : 0u, fnext = kEarlyStop ? ((it + 1) & 1) : 0u;
+        uint32_t& s_flag = s_flag2[fcur];
+        uint32_t& s_novf = s_novf2[fcur];
         if (threadIdx.x == 0) {
-            s_flag = 0;
-            s_novf = 0;
+            s_flag2[fnext] = 0;
+            s_novf2[fnext] = 0;
             s_nob = 0;
             s_pool = 0;
         }
@@ -617,7 +638,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                 const uint32_t i = atomicAdd(&s_novf, 1u);
                 if (i < OVCAP) ovl[i] = c; else s_flag = 1;
             }
-        });
+        }, kEarlyStop ? &s_flag : nullptr);
         PROBE(4);
         bool fallback = s_flag != 0;  // overflow list full: the row goes to the bitmap bin
         if (!fallback) {
