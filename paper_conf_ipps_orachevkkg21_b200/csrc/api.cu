@@ -81,7 +81,7 @@ spbla_Status spbla_Initialize(int device) {
             CUDA_CHECK(cudaMemPoolCreate(&c.mat_pool, &props));
             CUDA_CHECK(cudaMemPoolSetAttribute(c.mat_pool, cudaMemPoolAttrReleaseThreshold, &thr));
         }
-        CUDA_CHECK(cudaMallocHost(&c.host_words, 64));
+        CUDA_CHECK(cudaMallocHost(&c.host_words, 256));
         c.stream = 0;
         c.device = device;
     });

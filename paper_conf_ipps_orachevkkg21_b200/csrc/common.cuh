@@ -53,6 +53,8 @@ void dev_free(void* p, size_t bytes);
 // read `n` uint64 words from device memory (synchronises the stream)
 void trace_mark(const char* what);
 void read_words(const uint64_t* dev, uint64_t* host, int n);
+// read_words plus up to 128 more bytes from dev2 into host2, one synchronisation
+void read_words2(const uint64_t* dev, uint64_t* host, int n, const void* dev2, void* host2, size_t bytes2);
 void memset_async(void* p, int v, size_t bytes);
 void copy_async(void* dst, const void* src, size_t bytes, cudaMemcpyKind kind);
 inline void count_launch(int n = 1) { ctx().launches += n; }

@@ -98,6 +98,16 @@ void read_words(const uint64_t* dev, uint64_t* host, int n) {
     std::memcpy(host, g_ctx.host_words, n * sizeof(uint64_t));
 }
 
+void read_words2(const uint64_t* dev, uint64_t* host, int n, const void* dev2, void* host2, size_t bytes2) {
+    if (n > 8 || bytes2 > 128) throw Error(SPBLA_STATUS_INVALID_ARGUMENT, "read_words2: too many bytes");
+    unsigned char* hw = reinterpret_cast<unsigned char*>(g_ctx.host_words);
+    CUDA_CHECK(cudaMemcpyAsync(hw, dev, n * sizeof(uint64_t), cudaMemcpyDeviceToHost, g_ctx.stream));
+    CUDA_CHECK(cudaMemcpyAsync(hw + 128, dev2, bytes2, cudaMemcpyDeviceToHost, g_ctx.stream));
+    CUDA_CHECK(cudaStreamSynchronize(g_ctx.stream));
+    std::memcpy(host, hw, n * sizeof(uint64_t));
+    std::memcpy(host2, hw + 128, bytes2);
+}
+
 void memset_async(void* p, int v, size_t bytes) {
     if (bytes) CUDA_CHECK(cudaMemsetAsync(p, v, bytes, g_ctx.stream));
 }

@@ -1480,9 +1480,15 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     bin_scatter_kernel<<<gb, 256, 0, st>>>(bin.p, nrows, cursor, rows.p);
     count_launch();
     check_launch("bin_scatter_kernel");
+    // one synchronisation: the scratch size and the bin histogram (empty bins
+    // are not launched; small ones get only as many blocks as rows)
     uint64_t h[2];
-    read_words(soff.p + nrows, h, 1);
+    uint32_t hcnt[kNumBins];
+    read_words2(soff.p + nrows, h, 1, hist, hcnt, sizeof(hcnt));
     const uint64_t scratch_total = h[0];
+    auto grid_for = [&](int b, uint32_t full) { return std::min<uint32_t>(full, hcnt[b]); };
+    uint32_t hash_rows = 0;
+    for (int b = BIN_H0; b <= BIN_H6; ++b) hash_rows += hcnt[b];
     cap.release();
     bin.release();
     trace_mark("binning");
@@ -1500,17 +1506,24 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     //    out by an atomic work counter, so heavy rows balance dynamically)
     int t;
     t = ktime_begin("dense", st);
-    DENSE<<<nsm, 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols, scratch.p, soff.p,
-                                     counts.p, work);
+    if (hcnt[BIN_DENSE]) {
+        DENSE<<<grid_for(BIN_DENSE, nsm), 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols,
+                                                              scratch.p, soff.p, counts.p, work);
+        count_launch();
+    }
     ktime_end(t);
 #define LAUNCH_HASH(K, NAME, BIN, W)                                                                   \
     t = ktime_begin(#NAME, st);                                                                          \
-    if (src.kind == 0)                                                                                   \
-        K(0)<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p,    \
-                                                                counts.p, work + W, ovf_rows.p, ovf);   \
-    else                                                                                                 \
-        K(1)<<<nsm * NAME##_PERSM, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p,    \
-                                                                counts.p, work + W, ovf_rows.p, ovf);   \
+    if (hcnt[BIN]) {                                                                                     \
+        const uint32_t g = grid_for(BIN, uint32_t(nsm * NAME##_PERSM));                                  \
+        if (src.kind == 0)                                                                               \
+            K(0)<<<g, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p, counts.p, work + W, \
+                                                   ovf_rows.p, ovf);                                     \
+        else                                                                                             \
+            K(1)<<<g, NAME##_T, NAME##_SMEM, st>>>(src, recs.p, binoff + BIN, scratch.p, counts.p, work + W, \
+                                                   ovf_rows.p, ovf);                                     \
+        count_launch();                                                                                  \
+    }                                                                                                    \
     ktime_end(t);
     LAUNCH_HASH(HASH6, H6, BIN_H6, 7)
     LAUNCH_HASH(HASH5, H5, BIN_H5, 1)
@@ -1522,20 +1535,29 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
 #undef LAUNCH_HASH
     // rows whose hash probes ran long: bitmap path
     t = ktime_begin("dense_ovf", st);
-    SDENSE<<<nsm * 5, 256, kSDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work2);
-    DENSE<<<nsm, 1024, kDSmem, st>>>(src, ovf_rows.p, ovf + 2, range, ncols, scratch.p, soff.p, counts.p, work + 6);
+    if (hash_rows) {  // (fallback rows come only from the hash bins)
+        const uint32_t g = std::min<uint32_t>(nsm * 5, hash_rows);
+        SDENSE<<<g, 256, kSDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work2);
+        DENSE<<<std::min<uint32_t>(nsm, hash_rows), 1024, kDSmem, st>>>(src, ovf_rows.p, ovf + 2, range, ncols,
+                                                                        scratch.p, soff.p, counts.p, work + 6);
+        count_launch(2);
+    }
     ktime_end(t);
-    count_launch();
-    count_launch(9);
     check_launch("block bins");
     const unsigned gw = nsm * 8;  // 256-thread blocks, grid-stride over bin rows
     t = ktime_begin("warp_bins", st);
-    warp_bin_kernel<8><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W8, scratch.p, soff.p, counts.p);
-    warp_bin_kernel<4><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W4, scratch.p, soff.p, counts.p);
-    warp_bin_kernel<2><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W2, scratch.p, soff.p, counts.p);
-    warp_bin_kernel<1><<<gw, 256, 0, st>>>(src, rows.p, binoff, BIN_W1, scratch.p, soff.p, counts.p);
+#define LAUNCH_WARP(E, BIN)                                                                                \
+    if (hcnt[BIN]) {                                                                                     \
+        warp_bin_kernel<E><<<std::min<uint32_t>(gw, (hcnt[BIN] + 7) / 8), 256, 0, st>>>(src, rows.p, binoff, BIN, \
+                                                                                        scratch.p, soff.p, counts.p); \
+        count_launch();                                                                                  \
+    }
+    LAUNCH_WARP(8, BIN_W8)
+    LAUNCH_WARP(4, BIN_W4)
+    LAUNCH_WARP(2, BIN_W2)
+    LAUNCH_WARP(1, BIN_W1)
+#undef LAUNCH_WARP
     ktime_end(t);
-    count_launch(4);
     check_launch("warp_bin_kernel");
     trace_mark("bin kernels");
     // 5. row offsets
