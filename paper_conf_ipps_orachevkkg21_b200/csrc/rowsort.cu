@@ -952,38 +952,47 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                     if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
                 }
             });
-            // emission over the top level: warp w owns top words [w*tc, (w+1)*tc)
+            // emission over the top level: warp w owns top words [w*tc, (w+1)*tc),
+            // read 32 at a time (one per lane); a ballot gives the non-zero
+            // ones and the warp visits only those (rows of a few hundred
+            // columns leave most top words empty: the per-word loop was the
+            // kernel's largest instruction count)
             constexpr uint32_t tc = kTop / NW;
             const uint32_t tb = wib * tc;
             uint32_t cnt = 0;
-            for (uint32_t t = tb; t < tb + tc; ++t) {  // warp-uniform loop over top words
-                const uint32_t tw = top[t];
-                if (tw == 0) continue;
-                const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
-                cnt += __popc(word);
+            for (uint32_t t0 = tb; t0 < tb + tc; t0 += 32) {
+                const uint32_t tl = t0 + lane < tb + tc ? top[t0 + lane] : 0u;
+                for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {  // warp-uniform
+                    const uint32_t j = __ffs(m) - 1, t = t0 + j;
+                    const uint32_t tw = __shfl_sync(FULL, tl, j);
+                    const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                    cnt += __popc(word);
+                }
             }
             cnt = warp_sum(cnt);
             if (lane == 0) s_w[wib] = cnt;
             __syncthreads();
             scan_warp_counts<NW>(s_w);
             uint32_t pos = s_w[wib];
-            for (uint32_t t = tb; t < tb + tc; ++t) {
-                const uint32_t tw = top[t];
-                if (tw == 0) continue;
-                uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
-                if ((tw >> lane) & 1u) bm[t * 32 + lane] = 0u;  // clean for the next row/window
-                const uint32_t c = __popc(word);
-                const uint32_t inc = warp_inclusive_scan(c);
-                uint32_t o = pos + inc - c;
-                const uint64_t colbase = wlo + (uint64_t(t * 32 + lane) << 5);
-                while (word) {
-                    const int bit = __ffs(word) - 1;
-                    word &= word - 1;
-                    out[written + o++] = idx_t(colbase + bit);
+            for (uint32_t t0 = tb; t0 < tb + tc; t0 += 32) {
+                const uint32_t tl = t0 + lane < tb + tc ? top[t0 + lane] : 0u;
+                for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {
+                    const uint32_t j = __ffs(m) - 1, t = t0 + j;
+                    const uint32_t tw = __shfl_sync(FULL, tl, j);
+                    uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                    if ((tw >> lane) & 1u) bm[t * 32 + lane] = 0u;  // clean for the next row/window
+                    const uint32_t c = __popc(word);
+                    const uint32_t inc = warp_inclusive_scan(c);
+                    uint32_t o = pos + inc - c;
+                    const uint64_t colbase = wlo + (uint64_t(t * 32 + lane) << 5);
+                    while (word) {
+                        const int bit = __ffs(word) - 1;
+                        word &= word - 1;
+                        out[written + o++] = idx_t(colbase + bit);
+                    }
+                    pos += __shfl_sync(FULL, inc, 31);
                 }
-                pos += __shfl_sync(FULL, inc, 31);
-                __syncwarp();
-                if (lane == 0) top[t] = 0u;
+                if (tl) top[t0 + lane] = 0u;  // (each lane its own top word; tw came by shuffle)
             }
             written += s_w[32];
             __syncthreads();
