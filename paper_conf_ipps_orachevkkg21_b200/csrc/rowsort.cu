@@ -952,16 +952,19 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                     if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
                 }
             });
-            // emission over the top level: warp w owns top words [w*tc, (w+1)*tc),
+            // emission over the top level: warp w owns top words [tb, te),
             // read 32 at a time (one per lane); a ballot gives the non-zero
             // ones and the warp visits only those (rows of a few hundred
             // columns leave most top words empty: the per-word loop was the
             // kernel's largest instruction count)
-            constexpr uint32_t tc = kTop / NW;
-            const uint32_t tb = wib * tc;
+            // the window's used top words are split evenly over the warps
+            // (a fixed split left the warps outside the row's span idle)
+            const uint32_t used = uint32_t((whi - wlo + 1023) >> 10);
+            const uint32_t tcw = (used + NW - 1) / NW;
+            const uint32_t tb = min(used, wib * tcw), te = min(used, tb + tcw);
             uint32_t cnt = 0;
-            for (uint32_t t0 = tb; t0 < tb + tc; t0 += 32) {
-                const uint32_t tl = t0 + lane < tb + tc ? top[t0 + lane] : 0u;
+            for (uint32_t t0 = tb; t0 < te; t0 += 32) {
+                const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
                 for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {  // warp-uniform
                     const uint32_t j = __ffs(m) - 1, t = t0 + j;
                     const uint32_t tw = __shfl_sync(FULL, tl, j);
@@ -974,8 +977,8 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             __syncthreads();
             scan_warp_counts<NW>(s_w);
             uint32_t pos = s_w[wib];
-            for (uint32_t t0 = tb; t0 < tb + tc; t0 += 32) {
-                const uint32_t tl = t0 + lane < tb + tc ? top[t0 + lane] : 0u;
+            for (uint32_t t0 = tb; t0 < te; t0 += 32) {
+                const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
                 for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {
                     const uint32_t j = __ffs(m) - 1, t = t0 + j;
                     const uint32_t tw = __shfl_sync(FULL, tl, j);
