@@ -920,16 +920,35 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
     uint32_t* top = bm + kWords;
     __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
-    __shared__ uint32_t s_item;
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     fill_words(bm, kWords + kTop, 0u, THREADS);  // kept clean between rows
     __syncthreads();
-    for (;;) {
-        if (threadIdx.x == 0) s_item = bounds[0] + atomicAdd(work, 1u);
-        __syncthreads();
-        const uint32_t item = s_item;
-        if (item >= bounds[1]) break;
-        const idx_t r = rows[item];
+    // thread 0 claims a row one ahead and loads its row id during the
+    // current row (the claim and the id load left the block idle at every
+    // row start)
+    __shared__ uint32_t s_item2[2];
+    __shared__ idx_t s_r2[2];
+    const uint32_t lo_b = bounds[0], hi_b = bounds[1];
+    uint32_t c1 = 0;  // (thread 0) claimed item of the next row
+    if (threadIdx.x == 0) {
+        const uint32_t c0 = lo_b + atomicAdd(work, 1u);
+        s_item2[0] = c0;
+        if (c0 < hi_b) s_r2[0] = rows[c0];
+        c1 = c0 < hi_b ? lo_b + atomicAdd(work, 1u) : hi_b;
+    }
+    __syncthreads();
+#pragma unroll 1
+    for (uint32_t it = 0;; ++it) {
+        const uint32_t cur = it & 1u;
+        const uint32_t item = s_item2[cur];
+        if (item >= hi_b) break;
+        const idx_t r = s_r2[cur];
+        idx_t rn = 0;
+        uint32_t c2 = hi_b;
+        if (threadIdx.x == 0 && c1 < hi_b) {
+            rn = rows[c1];
+            c2 = lo_b + atomicAdd(work, 1u);
+        }
         uint32_t clo = 0, chi = ncols - 1;
         if (range) {
             const uint2 rg = range[r];
@@ -1000,7 +1019,13 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             written += s_w[32];
             __syncthreads();
         }
-        if (threadIdx.x == 0) counts[r] = written;
+        if (threadIdx.x == 0) {
+            counts[r] = written;
+            s_item2[cur ^ 1u] = c1;
+            s_r2[cur ^ 1u] = rn;
+            c1 = c2;
+        }
+        __syncthreads();
     }
 }
 
