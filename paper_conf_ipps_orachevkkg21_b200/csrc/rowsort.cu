@@ -906,7 +906,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
 // with > 40960 products) and 256 threads x 256 Ki-bit windows, 5 blocks per
 // SM (hash-bin rows that fell back - e.g. duplicate-heavy closure rows - and
 // whose span fits two windows).
-template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS>
+template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS, bool FCOUNT>
 __global__ void __launch_bounds__(THREADS)
 dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
                  const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
@@ -962,6 +962,15 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         for (uint32_t w = 0; w < nwin; ++w) {
             const uint64_t wlo = uint64_t(clo) + uint64_t(w) * BITS;
             const uint64_t whi = min(wlo + BITS, uint64_t(chi) + 1);
+            // the window's used top words are split evenly over the warps
+            // (a fixed split left the warps outside the row's span idle)
+            const uint32_t used = uint32_t((whi - wlo + 1023) >> 10);
+            const uint32_t tcw = (used + NW - 1) / NW;
+            const uint32_t tb = min(used, wib * tcw), te = min(used, tb + tcw);
+            // FCOUNT: every newly set bit is counted for its owner warp during
+            // the gather (s_w is clean before the gather's staging barrier),
+            // so the emission needs one walk instead of two
+            if (FCOUNT && threadIdx.x < NW) s_w[threadIdx.x] = 0u;
             block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH, false,
                                            [&](idx_t c) {
                 if (c >= wlo && c < whi) {
@@ -969,6 +978,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                     const uint32_t bit = 1u << (d & 31);
                     const uint32_t old = atomicOr(&bm[d >> 5], bit);
                     if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
+                    if (FCOUNT && !(old & bit)) atomicAdd(&s_w[(d >> 10) / tcw], 1u);
                 }
             });
             // emission over the top level: warp w owns top words [tb, te),
@@ -976,11 +986,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             // ones and the warp visits only those (rows of a few hundred
             // columns leave most top words empty: the per-word loop was the
             // kernel's largest instruction count)
-            // the window's used top words are split evenly over the warps
-            // (a fixed split left the warps outside the row's span idle)
-            const uint32_t used = uint32_t((whi - wlo + 1023) >> 10);
-            const uint32_t tcw = (used + NW - 1) / NW;
-            const uint32_t tb = min(used, wib * tcw), te = min(used, tb + tcw);
+            if (!FCOUNT) {
             uint32_t cnt = 0;
             for (uint32_t t0 = tb; t0 < te; t0 += 32) {
                 const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
@@ -994,6 +1000,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             cnt = warp_sum(cnt);
             if (lane == 0) s_w[wib] = cnt;
             __syncthreads();
+            }  // (FCOUNT: the gather ended with a barrier after the counts)
             scan_warp_counts<NW>(s_w);
             uint32_t pos = s_w[wib];
             for (uint32_t t0 = tb; t0 < te; t0 += 32) {
@@ -1450,11 +1457,11 @@ HBIN(H6, H6_CFG)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
 static_assert(kDSmem + 2048 <= 227 * 1024, "dense bin smem");
 static_assert((kDenseBits / 1024) % 32 == 0, "dense bin: top words per warp");
-#define DENSE dense_bin_kernel<1024, kDBatch, 8, kDenseBits>
+#define DENSE dense_bin_kernel<1024, kDBatch, 8, kDenseBits, false>
 constexpr uint32_t kSDenseBits = 1u << 18, kSDBatch = 256;
 constexpr size_t kSDSmem = kSDBatch * kSegBytes + (kSDenseBits / 32 + kSDenseBits / 1024) * sizeof(uint32_t);
 static_assert(5 * (kSDSmem + 2048) <= 228 * 1024, "small dense bin residency");
-#define SDENSE dense_bin_kernel<256, kSDBatch, 4, kSDenseBits>
+#define SDENSE dense_bin_kernel<256, kSDBatch, 4, kSDenseBits, true>
 
 static void ensure_attrs() {
     static int done_dev = -1;
