@@ -18,6 +18,6 @@ done
 ls -la $O
 # the other BASELINE rows: configs[2] (EWiseAdd + Kronecker) and configs[3] (closure)
 for wl in ewise_kron closure18; do
-  timeout 600 python bench.py --workload $wl --steps 5 > $O/bench_$wl.json 2> $O/bench_$wl.err
+  timeout 600 python bench.py --workload $wl --steps 9 --warmup 5 > $O/bench_$wl.json 2> $O/bench_$wl.err
 done
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:ewise_merge -s 3 -c 1 -o $O/top_ewise_merge -f python bench.py --workload ewise_kron --steps 1 --warmup 3 > $O/ncu_top_ewise.log 2>&1
