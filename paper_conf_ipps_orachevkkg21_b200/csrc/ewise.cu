@@ -29,9 +29,13 @@ namespace spbla {
 
 namespace {
 
-constexpr int kThreads = 256;
+#ifndef SPBLA_EW_THREADS  // (overridable for a sweep)
+#define SPBLA_EW_THREADS 512
+#endif
+constexpr int kThreads = SPBLA_EW_THREADS;
+constexpr int kMinBlocks = 1536 / kThreads;  // 1536 threads per SM at ~30 KB smem per 2048 items
 constexpr int kItems = 8;
-constexpr uint32_t kTile = kThreads * kItems;  // 2048 merged items per tile
+constexpr uint32_t kTile = kThreads * kItems;  // merged items per tile (4096 at 512 threads)
 // padded smem indices: threads own kItems consecutive positions, so a plain
 // layout puts the lanes of a warp kItems words apart (8- to 16-way bank
 // conflicts); one pad word per 16 (keys, 64-bit) / 32 (marks, output) words
@@ -101,7 +105,7 @@ __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
     return v;
 }
 
-__global__ void __launch_bounds__(kThreads, 6)
+__global__ void __launch_bounds__(kThreads, kMinBlocks)
 ewise_merge_kernel(MergeIn m, uint64_t ntiles, const uint32_t* __restrict__ tile_row,
                    const uint64_t* __restrict__ tile_a, const uint32_t* __restrict__ tile_rlo,
                    const uint64_t* __restrict__ tile_prev, uint64_t* status, uint32_t* ticket,
