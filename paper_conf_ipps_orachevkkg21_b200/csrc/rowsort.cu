@@ -918,7 +918,6 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
     uint32_t* bm = reinterpret_cast<uint32_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
     uint32_t* top = bm + kWords;
-    __shared__ uint64_t s_scan[33];
     __shared__ uint32_t s_w[33];
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     fill_words(bm, kWords + kTop, 0u, THREADS);  // kept clean between rows
@@ -986,21 +985,21 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             // ones and the warp visits only those (rows of a few hundred
             // columns leave most top words empty: the per-word loop was the
             // kernel's largest instruction count)
-            if (!FCOUNT) {
-            uint32_t cnt = 0;
-            for (uint32_t t0 = tb; t0 < te; t0 += 32) {
-                const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
-                for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {  // warp-uniform
-                    const uint32_t j = __ffs(m) - 1, t = t0 + j;
-                    const uint32_t tw = __shfl_sync(FULL, tl, j);
-                    const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
-                    cnt += __popc(word);
+            if (!FCOUNT) {  // (FCOUNT: the gather ended with a barrier after the counts)
+                uint32_t cnt = 0;
+                for (uint32_t t0 = tb; t0 < te; t0 += 32) {
+                    const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
+                    for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {  // warp-uniform
+                        const uint32_t j = __ffs(m) - 1, t = t0 + j;
+                        const uint32_t tw = __shfl_sync(FULL, tl, j);
+                        const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                        cnt += __popc(word);
+                    }
                 }
+                cnt = warp_sum(cnt);
+                if (lane == 0) s_w[wib] = cnt;
+                __syncthreads();
             }
-            cnt = warp_sum(cnt);
-            if (lane == 0) s_w[wib] = cnt;
-            __syncthreads();
-            }  // (FCOUNT: the gather ended with a barrier after the counts)
             scan_warp_counts<NW>(s_w);
             uint32_t pos = s_w[wib];
             for (uint32_t t0 = tb; t0 < te; t0 += 32) {
