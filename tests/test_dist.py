@@ -79,6 +79,12 @@ def worker(rank, world, port, q):
         Cl2, it = spdist.distributed_closure(ops, rows_of(G, s0, s1), m)
         ref, ref_it = oracle.closure(G)
         ok_clo = (Cl2 == rows_of(ref, s0, s1)) and it == ref_it
+        # degenerate split: rank 1 owns no rows (empty CSR block in the
+        # padded all-gather, 0-row local multiply)
+        eb = [0, n, n]
+        Ae = rows_of(A, eb[rank], eb[rank + 1])
+        Ce = spdist.distributed_mxm(ops, Ae, Ae, n, n)
+        ok_mxm = ok_mxm and Ce == rows_of(full, eb[rank], eb[rank + 1])
         q.put((rank, bool(ok_mxm), bool(ok_clo), bounds, it, ref_it))
     finally:
         dist.destroy_process_group()
