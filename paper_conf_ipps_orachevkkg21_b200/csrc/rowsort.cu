@@ -1457,9 +1457,10 @@ constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 
 static_assert(kDSmem + 2048 <= 227 * 1024, "dense bin smem");
 static_assert((kDenseBits / 1024) % 32 == 0, "dense bin: top words per warp");
 #define DENSE dense_bin_kernel<1024, kDBatch, 8, kDenseBits, false>
-constexpr uint32_t kSDenseBits = 1u << 18, kSDBatch = 256;
+constexpr uint32_t kSDenseBits = 1u << 18, kSDBatch = 192;
+constexpr int kSDPerSM = 6;  // blocks per SM (the kernel is barrier/latency-bound: residency pays)
 constexpr size_t kSDSmem = kSDBatch * kSegBytes + (kSDenseBits / 32 + kSDenseBits / 1024) * sizeof(uint32_t);
-static_assert(5 * (kSDSmem + 2048) <= 228 * 1024, "small dense bin residency");
+static_assert(kSDPerSM * (kSDSmem + 1024 + 512) <= 228 * 1024, "small dense bin residency");
 #define SDENSE dense_bin_kernel<256, kSDBatch, 4, kSDenseBits, true>
 
 static void ensure_attrs() {
@@ -1579,7 +1580,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     // rows whose hash probes ran long: bitmap path
     t = ktime_begin("dense_ovf", st);
     if (hash_rows) {  // (fallback rows come only from the hash bins)
-        const uint32_t g = std::min<uint32_t>(nsm * 5, hash_rows);
+        const uint32_t g = std::min<uint32_t>(nsm * kSDPerSM, hash_rows);
         SDENSE<<<g, 256, kSDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work2);
         DENSE<<<std::min<uint32_t>(nsm, hash_rows), 1024, kDSmem, st>>>(src, ovf_rows.p, ovf + 2, range, ncols,
                                                                         scratch.p, soff.p, counts.p, work + 6);
