@@ -903,7 +903,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
 // top bit t set <=> bm word t may be non-zero.  Emission walks the top level,
 // so clearing and emitting cost O(words touched + BITS/1024).  Two configs:
 // 1024 threads x 1.5 Mi-bit windows, one block per SM (the dense bin: rows
-// with > 40960 products) and 256 threads x 256 Ki-bit windows, 5 blocks per
+// with > 40960 products) and 256 threads x 256 Ki-bit windows, 6 blocks per
 // SM (hash-bin rows that fell back - e.g. duplicate-heavy closure rows - and
 // whose span fits two windows).
 template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS, bool FCOUNT>
