@@ -25,8 +25,8 @@
  *  - All device work is enqueued on the library stream (spbla_SetStream; the
  *    legacy default stream until set).  Entry points that must learn a result
  *    size on the host (Build, MxM, EWiseAdd, Transpose, ExtractSubMatrix,
- *    Reduce, TransitiveClosure, AssembleRowBlocks) synchronise that stream once
- *    or twice; all others are asynchronous.
+ *    Reduce, TransitiveClosure) synchronise that stream once or twice; all
+ *    others (AssembleRowBlocks included) are asynchronous.
  *  - Pointer arguments flagged with SPBLA_HINT_HOST_MEMORY are host memory;
  *    otherwise they are device memory of the current device.  Caller-owned
  *    buffers stay caller-owned; matrices own their storage unless created by
@@ -79,7 +79,10 @@ typedef enum {
 spbla_Status spbla_Initialize(int device);
 /* Free pooled memory; matrices must have been freed. */
 spbla_Status spbla_Finalize(void);
-/* Enqueue all further work on `stream` (a cudaStream_t, may be 0). */
+/* Enqueue all further work on `stream` (a cudaStream_t, may be 0).  When
+ * the stream changes, the new stream first waits (an event) for all work
+ * already queued on the old one, so matrices and pooled scratch still in use
+ * there are never reused early. */
 spbla_Status spbla_SetStream(void* stream);
 spbla_Status spbla_GetStream(void** stream);
 /* Synchronise the library stream. */

@@ -105,7 +105,19 @@ spbla_Status spbla_Finalize(void) {
 spbla_Status spbla_SetStream(void* stream) {
     return guarded([&] {
         require_init();
-        ctx().stream = (cudaStream_t)stream;
+        Context& c = ctx();
+        cudaStream_t ns = (cudaStream_t)stream;
+        if (ns != c.stream) {
+            // work already queued on the old stream (and the stream-ordered
+            // frees of storage it uses) must precede everything issued on the
+            // new one: the new stream waits for the old stream's tail
+            cudaEvent_t ev;
+            CUDA_CHECK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+            CUDA_CHECK(cudaEventRecord(ev, c.stream));
+            CUDA_CHECK(cudaStreamWaitEvent(ns, ev, 0));
+            CUDA_CHECK(cudaEventDestroy(ev));
+        }
+        c.stream = ns;
     });
 }
 

@@ -571,8 +571,9 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             have_nx = nxt1 < hi_i;
             if (have_nx) nx = recs[nxt1];
         }
-        // (single-buffered in the bins without the early stop, as before)
-        const uint32_t fcur = kEarlyStop ? (it & 1) : 0u, fnext = kEarlyStop ? ((it + 1) & 1) : 0u;
+        // row-parity pair in every bin: the gather may start before thread 0
+        // reaches this point, so a row never clears its own flag/counter
+        const uint32_t fcur = it & 1u, fnext = (it + 1) & 1u;
         uint32_t& s_flag = s_flag2[fcur];
         uint32_t& s_novf = s_novf2[fcur];
         if (threadIdx.x == 0) {
@@ -816,8 +817,10 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                 const uint32_t jn = min(32u, np - mb);
 #pragma unroll 1
                 for (uint32_t j = 0; j < jn; j += 8) {
-                    // past the last pair a lane group repeats pair mb+j and stores
-                    // nothing (its restores write the same clean values)
+                    // past the last pair a lane group repeats pair mb+j read-only:
+                    // it neither stores columns nor restores table words (the
+                    // owning group g4 = 0 restores them; no intra-warp
+                    // read/write overlap)
                     const bool ok = j + g4 < jn;
                     const uint32_t m = mb + j + (ok ? g4 : 0u);
                     uint32_t* wp = tabw + (4 * t8) * MPP + m;
@@ -825,7 +828,8 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
 #pragma unroll
                     for (int k = 0; k < 4; ++k) wv[k] = wp[k * MPP];
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) wp[k * MPP] = 0xFFFFFFFFu;
+                    for (int k = 0; k < 4; ++k)
+                        if (ok) wp[k * MPP] = 0xFFFFFFFFu;
                     uint32_t inc[4], ex;
                     if (DEDUP_B) {
                         uint32_t prevw = __shfl_up_sync(FULL, wv[3], 1, 4);
