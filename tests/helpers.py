@@ -52,3 +52,42 @@ def csr_is_valid(rp, ci, ncols):
     starts = rp[:-1][np.diff(rp) > 0]
     row_start[starts] = True
     return bool(np.all((d > 0) | row_start[1:]))
+
+
+def dag_reach_and_depth(n, src, dst):
+    """Reachability (paths of length >= 1) and the longest shortest-path
+    length D of a DAG whose edges v -> u all have u < v: processing v in
+    increasing order, reach(v) = U_{u in out(v)} ({u} U reach(u)) with
+    dist_v(w) = 1 + min over those u (0 for w = u itself).  Independent of the
+    oracle and of the CUDA path (a different algorithm than C += C.C)."""
+    src = np.asarray(src, np.int64)
+    dst = np.asarray(dst, np.int64)
+    assert np.all(dst < src), "labeled_dag edges point to smaller ids"
+    o = np.argsort(src, kind="stable")
+    d = dst[o]
+    st = np.searchsorted(src[o], np.arange(n + 1))
+    reach, dist = [None] * n, [None] * n
+    empty_t, empty_d = np.zeros(0, np.int64), np.zeros(0, np.int32)
+    D = 0
+    for v in range(n):
+        kids = d[st[v]:st[v + 1]]
+        if len(kids) == 0:
+            reach[v], dist[v] = empty_t, empty_d
+            continue
+        pt, pd = [kids], [np.ones(len(kids), np.int32)]
+        for u in kids.tolist():
+            pt.append(reach[u])
+            pd.append(dist[u] + 1)
+        t = np.concatenate(pt)
+        dd = np.concatenate(pd)
+        oo = np.lexsort((dd, t))
+        t, dd = t[oo], dd[oo]
+        first = np.empty(len(t), bool)
+        first[0] = True
+        first[1:] = t[1:] != t[:-1]
+        reach[v], dist[v] = t[first], dd[first]
+        D = max(D, int(dist[v].max()))
+    lens = np.array([len(x) for x in reach], np.int64)
+    rp = np.zeros(n + 1, np.uint64)
+    rp[1:] = np.cumsum(lens)
+    return oracle.Csr(n, n, rp, np.concatenate(reach).astype(np.uint32)), D

@@ -1,9 +1,22 @@
-"""BASELINE.json configs at full size, in the launch configuration bench.py
-times: the CUDA result is checked on sampled rows against the oracle computed
-row by row (heaviest rows and a representative of every bin included), and
-for all rows by properties that hold at any size (CSR invariants on the
-device, nnz and row counts)."""
-import collections
+"""BASELINE.json configs at FULL size, in the launch configuration bench.py
+times, compared bit for bit over EVERY row:
+
+* configs[1] / configs[4] (A.A on R-MAT 2^20 / 2^22): A built by the CUDA
+  Matrix_Build against the unchanged oracle's build (row blocks on all host
+  cores), then C = A.A against the unchanged oracle's ``mxm_rows`` over row
+  chunks on all host cores (``oracle/parallel.py``: ctypes releases the GIL,
+  so a thread pool is truly parallel).  Every rowptr entry and every column
+  of C is compared.  configs[1] also checks C += A.A (accumulate) the same way.
+* configs[3] (closure of the 2^18-vertex labelled DAG): the whole closure
+  CSR against reachability computed by an independent dynamic program over
+  the DAG (edges point to smaller ids, so vertices in increasing order see
+  their successors' closures complete), and the exact iteration count of the
+  C += C.C loop from the same DP's longest shortest-path length D: after k
+  evaluations C holds the paths of length 1..2^k, and the loop stops at the
+  first evaluation that adds nothing, k* = ceil(log2 D) + 1 (R9).
+* configs[2] (EWiseAdd 2^20 + Kronecker 2^10 (x) 64): whole CSR vs the oracle.
+"""
+import threading
 
 import numpy as np
 import pytest
@@ -11,7 +24,8 @@ import torch
 
 import oracle
 import spgen
-from helpers import assert_same, gpu_lib
+from oracle import parallel as par
+from helpers import assert_same, dag_reach_and_depth, gpu_lib
 
 pytestmark = pytest.mark.gpu
 
@@ -21,70 +35,78 @@ def sp():
     return gpu_lib()
 
 
-def host_csr(M):
-    rp, ci = M.to_csr()
-    return oracle.Csr(M.nrows, M.ncols, rp, ci)
-
-
-def check_rows(C, A, rows, Cin=None):
-    """C's rows `rows` equal the oracle's (C_in +) A.A rows, bit for bit."""
-    Ah = host_csr(A)
-    want = oracle.mxm_rows(Ah, Ah, rows, host_csr(Cin) if Cin is not None else None)
-    rp, ci = C.device_tensors()
-    rows_t = torch.as_tensor(rows.astype(np.int64), device="cuda")
-    b, e = rp[rows_t].cpu().numpy(), rp[rows_t + 1].cpu().numpy()
-    ci_h = ci.cpu().numpy().astype(np.uint32) if C.nvals < (1 << 31) else None
-    for t, r in enumerate(rows):
-        got = (ci_h[b[t]:e[t]] if ci_h is not None else ci[int(b[t]):int(e[t])].cpu().numpy().astype(np.uint32))
-        exp = want.colidx[int(want.rowptr[t]):int(want.rowptr[t + 1])]
-        assert np.array_equal(got, exp), f"row {r}: {len(got)} vs {len(exp)} entries"
-
-
-def sample_rows(ub, n, k=300, seed=0):
-    rng = np.random.default_rng(seed)
-    ub_h = ub.cpu().numpy()
-    heavy = np.argsort(ub_h)[-20:]
-    edges = [0, 1, 33, 65, 129, 257, 513, 1025, 2049, 4097, 8193, 20481, 40961, 1 << 62]
-    per_bin = []
-    for lo, hi in zip(edges[:-1], edges[1:]):
-        idx = np.nonzero((ub_h >= lo) & (ub_h < hi))[0]
-        if len(idx):
-            per_bin.append(rng.choice(idx, min(10, len(idx)), replace=False))
-    rnd = rng.integers(0, n, k)
-    return np.unique(np.concatenate([heavy, rnd, *per_bin, [0, n - 1]])).astype(np.uint32)
-
-
-def ub_of(A):
-    rp, ci = A.device_tensors()
-    lens = rp[1:] - rp[:-1]
-    rows = torch.repeat_interleave(torch.arange(A.nrows, device="cuda"), lens)
-    return torch.zeros(A.nrows, dtype=torch.int64, device="cuda").index_add_(0, rows, lens[ci.long()])
-
-
 def validate_on_device(sp, M):
     rp, ci = M.device_tensors()
     sp.Matrix.wrap(M.nrows, M.ncols, rp, ci, hints=sp.HINT_VALIDATE).free()  # raises on violation
 
 
+def compare_csr_chunked(C, want_rows, chunks):
+    """Every row of device matrix C against want_rows(r0, r1) -> oracle Csr of
+    rows [r0, r1), chunk by chunk on all host cores.  Returns nnz checked."""
+    rp_d, ci_d = C.device_tensors()
+    rp = rp_d.cpu().numpy().view(np.uint64)
+    assert rp[0] == 0 and int(rp[-1]) == C.nvals
+    errs, lk = [], threading.Lock()
+    checked = [0]
+
+    def one(r0, r1):
+        R = want_rows(r0, r1)
+        b, e = int(rp[r0]), int(rp[r1])
+        msg = None
+        if not np.array_equal(R.rowptr + np.uint64(b), rp[r0:r1 + 1]):
+            bad = np.nonzero(R.rowptr + np.uint64(b) != rp[r0:r1 + 1])[0][0]
+            msg = f"rowptr differs first at row {r0 + bad}"
+        else:
+            got = ci_d[b:e].cpu().numpy().view(np.uint32)
+            if not np.array_equal(got, R.colidx):
+                bad = np.nonzero(got != R.colidx)[0][0]
+                row = r0 + int(np.searchsorted(R.rowptr, bad, side="right")) - 1
+                msg = f"colidx differs first at position {b + bad} (row {row})"
+        with lk:
+            checked[0] += R.nvals
+            if msg:
+                errs.append(msg)
+
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=par.host_cores()) as ex:
+        list(ex.map(lambda ch: one(*ch), chunks))
+    assert not errs, f"{len(errs)} chunks differ: {errs[:3]}"
+    assert checked[0] == C.nvals
+    return checked[0]
+
+
+def mxm_chunks(Ah, Bh):
+    w = par.row_products(Ah, Bh)
+    return par.chunk_bounds(w, max(float(w.sum()) / (par.host_cores() * 24), 1e6))
+
+
 @pytest.mark.parametrize("wl", ["rmat20_ef16", "rmat22_ef32"])
-def test_mxm_full_size_sampled(sp, wl):
+def test_mxm_full_size_exact(sp, wl):
     import bench
     cfg = bench.WORKLOADS[wl]
-    n, r, c = bench.gen_pairs(cfg, "cuda")
+    n, r, c = bench.gen_pairs(cfg, "cuda")  # seeded generator (bit-identical on CPU and GPU)
     A = sp.Matrix.from_pairs(n, n, r, c)
+    Ah = par.build_chunked(n, n, r.cpu().numpy(), c.cpu().numpy())
     del r, c
-    ub = ub_of(A)
+    torch.cuda.empty_cache()
+    compare_csr_chunked(A, lambda r0, r1: oracle.Csr(
+        r1 - r0, n, Ah.rowptr[r0:r1 + 1] - Ah.rowptr[r0], Ah.colidx[int(Ah.rowptr[r0]):int(Ah.rowptr[r1])]),
+        par.chunk_bounds(np.diff(Ah.rowptr.astype(np.int64)), 4e6))
     C = sp.mxm(A, A)
     validate_on_device(sp, C)
-    assert C.nvals <= int(ub.sum())
-    rows = sample_rows(ub, n)
-    check_rows(C, A, rows)
+    chunks = mxm_chunks(Ah, Ah)
+    nnz = compare_csr_chunked(C, lambda r0, r1: oracle.mxm_rows(Ah, Ah, np.arange(r0, r1, dtype=np.uint32)),
+                              chunks)
+    print(f"{wl}: nnz(A) {Ah.nvals}, nnz(A.A) {nnz}: every row bit-exact vs the oracle")
     C.free()
-    if wl == "rmat20_ef16":  # accumulate in the same configuration
+    if wl == "rmat20_ef16":  # C += A.A (accumulate, C = A) in the same configuration
         Cacc = A.duplicate()
         sp.MxM(Cacc, A, A, accumulate=True)
         validate_on_device(sp, Cacc)
-        check_rows(Cacc, A, rows[:120], Cin=A)
+        compare_csr_chunked(Cacc, lambda r0, r1: oracle.mxm_rows(Ah, Ah, np.arange(r0, r1, dtype=np.uint32), Ah),
+                            chunks)
+        Cacc.free()
+    A.free()
 
 
 def test_ewise_kron_config2_full(sp):
@@ -94,9 +116,10 @@ def test_ewise_kron_config2_full(sp):
     A = sp.Matrix.from_pairs(n, n, r1.cuda(), c1.cuda())
     B = sp.Matrix.from_pairs(n, n, r2.cuda(), c2.cuda())
     E = sp.ewise_add(A, B)
-    OA = oracle.build(n, n, r1.numpy(), c1.numpy())
-    OB = oracle.build(n, n, r2.numpy(), c2.numpy())
+    OA = par.build_chunked(n, n, r1.numpy(), c1.numpy())
+    OB = par.build_chunked(n, n, r2.numpy(), c2.numpy())
     assert_same(A, OA, "A")
+    assert_same(B, OB, "B")
     assert_same(E, oracle.ewise_add(OA, OB), "A+B full")
     rg, cg = spgen.rmat_pairs(10, 16, 0.45, 0.22, 0.22, seed=3)
     rr, cr = spgen.rsm_pairs(64, 1, 2, seed=4)
@@ -107,9 +130,9 @@ def test_ewise_kron_config2_full(sp):
                                     oracle.build(64, 64, rr.numpy(), cr.numpy())), "G(x)R full")
 
 
-def test_closure_config3_full_sampled(sp):
-    """configs[3]: closure of a 2^18-vertex edge-labelled DAG; sampled rows
-    against BFS reachability (paths of length >= 1)."""
+def test_closure_config3_full_exact(sp):
+    """configs[3]: the whole closure CSR of the 2^18-vertex edge-labelled DAG
+    and the exact number of C += C.C evaluations."""
     n = 1 << 18
     (a0, b0), (a1, b1) = spgen.labeled_dag(n, 0.25, seed=9)
     L0 = sp.Matrix.from_pairs(n, n, a0.cuda(), b0.cuda())
@@ -117,20 +140,9 @@ def test_closure_config3_full_sampled(sp):
     U = sp.ewise_add(L0, L1)
     C, it = sp.closure(U)
     validate_on_device(sp, C)
-    assert 2 <= it <= 40
-    adj = collections.defaultdict(list)
-    for x, y in zip(np.concatenate([a0.numpy(), a1.numpy()]).tolist(),
-                    np.concatenate([b0.numpy(), b1.numpy()]).tolist()):
-        adj[x].append(y)
-    rp, ci = C.to_csr()
-    rng = np.random.default_rng(1)
-    for s in list(rng.integers(0, n, 150)) + [n - 1, 0]:
-        seen, st = set(), list(adj[int(s)])
-        while st:
-            v = st.pop()
-            if v in seen:
-                continue
-            seen.add(v)
-            st.extend(adj[v])
-        got = ci[int(rp[s]):int(rp[s + 1])]
-        assert np.array_equal(got, np.array(sorted(seen), dtype=np.uint32)), f"source {s}"
+    want, D = dag_reach_and_depth(n, np.concatenate([a0.numpy(), a1.numpy()]),
+                                  np.concatenate([b0.numpy(), b1.numpy()]))
+    assert_same(C, want, "closure(configs[3]) vs DAG reachability")
+    k_star = int(np.ceil(np.log2(D))) + 1 if D > 1 else 1
+    assert it == k_star, f"iterations {it}, expected ceil(log2 {D}) + 1 = {k_star}"
+    print(f"closure: nnz {C.nvals}, D = {D}, {it} evaluations")

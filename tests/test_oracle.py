@@ -340,3 +340,46 @@ def test_generator_deterministic_and_in_range():
     # power-law: max out-degree far above the mean
     deg = torch.bincount(r1.long(), minlength=1024)
     assert deg.max() > 4 * deg.float().mean()
+
+
+def test_parallel_driver_matches_serial_oracle():
+    """oracle/parallel.py only chunks rows: its results equal the serial oracle."""
+    import threading
+    from oracle import parallel as par
+    n = 1 << 12
+    r, c = spgen.rmat_pairs(12, 8, 0.45, 0.22, 0.22, seed=7)
+    A = oracle.build(n, n, r.numpy(), c.numpy())
+    assert par.build_chunked(n, n, r.numpy(), c.numpy(), block_rows=300, threads=4) == A
+    want = oracle.mxm(A, A, A)
+    w = par.row_products(A, A)
+    ch = par.chunk_bounds(w, float(w.sum()) / 13)
+    assert ch[0][0] == 0 and ch[-1][1] == n and all(a[1] == b[0] for a, b in zip(ch[:-1], ch[1:]))
+    got = {}
+    lk = threading.Lock()
+
+    def keep(r0, r1, R):
+        with lk:
+            got[r0] = R
+    par.mxm_rows_chunked(A, A, ch, keep, c=A, threads=4)
+    rp = [np.zeros(1, np.uint64)]
+    base = np.uint64(0)
+    for r0, _ in ch:
+        rp.append(got[r0].rowptr[1:] + base)
+        base += np.uint64(got[r0].nvals)
+    assert np.array_equal(np.concatenate(rp), want.rowptr)
+    assert np.array_equal(np.concatenate([got[r0].colidx for r0, _ in ch]), want.colidx)
+
+
+@pytest.mark.parametrize("n,p,seed", [(1500, 0.25, 9), (3000, 0.6, 2)])
+def test_dag_dp_matches_oracle_closure(n, p, seed):
+    """The full-size closure check's independent DAG dynamic program agrees
+    with the oracle's C += C.C loop, including the iteration count
+    ceil(log2 D) + 1 (R9)."""
+    from helpers import dag_reach_and_depth
+    (a0, b0), (a1, b1) = spgen.labeled_dag(n, p, seed=seed)
+    src = np.concatenate([a0.numpy(), a1.numpy()])
+    dst = np.concatenate([b0.numpy(), b1.numpy()])
+    want, it = oracle.closure(oracle.build(n, n, src, dst))
+    got, D = dag_reach_and_depth(n, src, dst)
+    assert got == want
+    assert it == int(np.ceil(np.log2(D))) + 1
