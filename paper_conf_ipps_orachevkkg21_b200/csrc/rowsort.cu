@@ -169,11 +169,12 @@ __device__ __forceinline__ void stage_one(const uint4& e, uint32_t i, uint32_t b
             sd_first[j] = i;
     }
 }
-template <int THREADS>
+// KINDT >= 0: the segment-source kind as a compile-time constant
+template <int THREADS, int KINDT = -1>
 __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint64_t sbase, uint32_t s0,
                                                    uint32_t n, const idx_t** sd_ptr, uint32_t* sd_end,
                                                    uint32_t* sd_first) {
-    if (s.kind == 1) {  // one segment
+    if ((KINDT >= 0 ? KINDT : s.kind) == 1) {  // one segment
         if (threadIdx.x == 0) {
             const off_t64 b = s.lrp[r];
             sd_ptr[0] = s.lst + b;
@@ -201,7 +202,7 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
 // is set every thread skips the rest of its products (the caller discards
 // the row).
 // prestaged: the first batch is already staged (and visible to all threads).
-template <int THREADS, int U, typename F>
+template <int THREADS, int U, int KINDT = -1, typename F>
 __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint64_t sbase, uint32_t nseg,
                                                const idx_t** sd_ptr, uint32_t* sd_end, uint32_t* sd_first,
                                                uint32_t batch, bool prestaged, F&& f,
@@ -210,7 +211,7 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
         const uint32_t ns = min(batch, nseg - s0);
         const uint32_t total = (s0 == 0 && prestaged)
                                    ? sd_end[ns - 1]
-                                   : stage_segments<THREADS>(s, r, sbase, s0, ns, sd_ptr, sd_end, sd_first);
+                                   : stage_segments<THREADS, KINDT>(s, r, sbase, s0, ns, sd_ptr, sd_end, sd_first);
 #ifdef SPBLA_PROBE
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
@@ -219,7 +220,7 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
             // thread: no barrier inside this loop)
             if (abort && *abort) break;
             uint32_t k;
-            if (s.kind == 1) {
+            if ((KINDT >= 0 ? KINDT : s.kind) == 1) {
                 k = 0;
             } else if (sd_first) {
                 k = sd_first[q0 >> kFirstShift];
