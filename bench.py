@@ -138,20 +138,32 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------------------
-def cpu_oracle_sample(rp_host, ci_host, ub_host, target_products):
-    """Time the CPU oracle (as it stands) on every k-th row of the workload."""
+def cpu_oracle_sample(rp_host, ci_host, ub_host, target_products, threads=None):
+    """Time the CPU oracle (as it stands: ``oracle.mxm_rows``) on a bounded
+    sample of the workload, on every host core: 4 contiguous row chunks per
+    thread spread evenly over the rows (oracle/parallel.py; ctypes releases
+    the GIL).  Returns (products, seconds, rows, threads, nnz)."""
     import numpy as np
     import oracle
+    from oracle import parallel as opar
+    threads = threads or opar.host_cores()
     n = len(rp_host) - 1
-    total = int(ub_host.sum())
-    k = max(1, int(np.ceil(total / target_products)))
-    rows = np.arange(0, n, k, dtype=np.uint32)
-    prods = int(ub_host[rows.astype(np.int64)].sum())
     A = oracle.Csr(n, n, rp_host, ci_host)
+    nch = 4 * threads
+    per = target_products / nch
+    cum = np.cumsum(ub_host.astype(np.float64))
+    total = float(cum[-1]) if n else 0.0
+    chunks = []
+    for i in range(nch):  # chunk i starts at the row holding product (i + 0.5) / nch of the total
+        r0 = int(np.searchsorted(cum, total * (i + 0.5) / nch))
+        r1 = int(np.searchsorted(cum, cum[min(r0, n - 1)] + per)) + 1
+        chunks.append((min(r0, n), min(max(r1, r0 + 1), n)))
+    prods = sum(int(ub_host[a:b].sum()) for a, b in chunks)
+    rows = sum(b - a for a, b in chunks)
     t = time.perf_counter()
-    out = oracle.mxm_rows(A, A, rows)
+    nnz = sum(opar.mxm_rows_chunked(A, A, chunks, lambda r0, r1, R: R.nvals, threads=threads))
     dt = time.perf_counter() - t
-    return prods, dt, len(rows), k, out.nvals
+    return prods, dt, rows, threads, nnz
 
 
 def run_reference(args):
@@ -175,44 +187,38 @@ def run_reference(args):
     rp_h = rp.cpu().numpy().astype(np.uint64)
     ci_h = ci.cpu().numpy().astype(np.uint32)
     ub = ub.cpu().numpy()
-    target = float(os.environ.get("REF_SAMPLE_PRODUCTS", "3e7"))
+    target = float(os.environ.get("REF_SAMPLE_PRODUCTS", "2e8"))
     times, prods = [], 0
     for i in range(args.warmup + args.steps):
-        p, dt, nrows, k, _ = cpu_oracle_sample(rp_h, ci_h, ub, target)
+        p, dt, nrows, thr, _ = cpu_oracle_sample(rp_h, ci_h, ub, target)
         if i >= args.warmup:
             times.append(dt)
             prods = p
     ms = 1e3 * sum(times) / len(times)
     value = prods / (ms * 1e-3) / 1e9
-    sample = f"every {k}-th row ({nrows} rows, {prods} products) of {args.workload}, std::set Gustavson, 1 thread"
+    sample = (f"{4 * thr} contiguous row chunks spread over {args.workload} ({nrows} rows, {prods} products); "
+              f"the unchanged std::set Gustavson oracle on {thr} threads")
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": args.workload, "baseline_config": wl["config"]},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": thr, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 
 # ---------------------------------------------------------------------------
-def run_aux(args):
-    """configs[2] (EWiseAdd 2^20 rows, Kronecker 2^10 graph x 64-state RSM) and
-    configs[3] (closure of a 2^18-vertex labelled DAG): device-timed with CUDA
-    events on the library stream, L2 flushed between steps; one JSON line.
-    1 GPU (these rows are replicas-only at N > 1)."""
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
-        return
-    import paper_conf_ipps_orachevkkg21_b200 as sp
-    torch.cuda.set_device(0)
-    sp.Initialize(0)
+AUX_GROUPS = ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "dense_ovf", "compact")
+
+
+def aux_timer(sp, steps, warmup):
+    """Device timing of a host-launched op (CUDA events on the library
+    stream, 256 MB L2 flush before each step); returns (timed, state) where
+    timed(fn) -> median ms and state collects launches and step lists."""
     stream = torch.cuda.current_stream()
-    peak_gbs, peak_src = load_peaks()
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device="cuda")
-    steps, warmup = args.steps, max(args.warmup, 3)
-    launches = []
-    step_lists = []
+    state = {"launches": 0, "step_ms": []}
 
     def timed(fn):
         for i in range(warmup):
@@ -232,78 +238,114 @@ def run_aux(args):
             e1.record(stream)
             e1.synchronize()
             ms.append(e0.elapsed_time(e1))
-        launches.append(sp.launch_count())
+        state["launches"] += sp.launch_count()
         log(f"[aux] step ms: {[round(x, 2) for x in ms]}")
-        step_lists.append([round(x, 3) for x in ms])
-        # median: these host-launch-bound ops see occasional 10-200 ms host
-        # stalls in pool allocations; the full list is reported
+        state["step_ms"].append([round(x, 3) for x in ms])
+        # median: these host-launched ops can see rare host stalls; the full
+        # list is reported next to it
         return statistics.median(ms)
+    return timed, state
 
+
+def aux_ewise_kron(sp, steps, warmup, peak_gbs):
+    """configs[2]: EWiseAdd of two 2^20-row matrices and Kronecker of a
+    2^10-vertex graph with a 64-state RSM adjacency."""
+    timed, state = aux_timer(sp, steps, warmup)
+    n = 1 << 20
+    r1, c1 = spgen.rmat_pairs(20, 16, 0.45, 0.22, 0.22, seed=1, device="cuda")
+    r2, c2 = spgen.uniform_pairs(n, n, 8, seed=2, device="cuda")
+    A = sp.Matrix.from_pairs(n, n, r1, c1)
+    B = sp.Matrix.from_pairs(n, n, r2, c2)
+    del r1, c1, r2, c2
+    E = sp.Matrix.new(n, n)
+    ms_e = timed(lambda: sp.Matrix_EWiseAdd(E, A, B))
+    ke = {k: sp.kernel_timing(k) for k in ("ewise_split", "ewise_merge")}
+    sp.set_kernel_timing(False)
+    # algorithmic bytes: both inputs read once (colidx + rowptr), output written once
+    alg_e = 4 * (A.nvals + B.nvals) + 16 * (n + 1) + 4 * E.nvals + 8 * (n + 1)
+    rg, cg = spgen.rmat_pairs(10, 16, 0.45, 0.22, 0.22, seed=3, device="cuda")
+    rr, cr = spgen.rsm_pairs(64, 1, 2, seed=4, device="cuda")
+    G = sp.Matrix.from_pairs(1024, 1024, rg, cg)
+    R = sp.Matrix.from_pairs(64, 64, rr, cr)
+    K = sp.Matrix.new(1024 * 64, 1024 * 64)
+    ms_k = timed(lambda: sp.Kronecker(K, G, R))
+    kk = sp.kernel_timing("kron")
+    sp.set_kernel_timing(False)
+    alg_k = 4 * K.nvals + 8 * (K.nrows + 1)  # output-write bound (inputs are KB)
+    per_e = (ke["ewise_split"][0] + ke["ewise_merge"][0]) / steps
+    out = {"ms": ms_e + ms_k, "unit": "ms",
+           "ewise": {"ms": ms_e, "kernel_ms": per_e, "nnz_A": A.nvals, "nnz_B": B.nvals, "nnz_C": E.nvals,
+                     "alg_bytes": alg_e, "GB/s": alg_e / (per_e * 1e-3) / 1e9,
+                     "frac": alg_e / (per_e * 1e-3) / 1e9 / peak_gbs,
+                     "kernel_ms_per_step": {k: v[0] / steps for k, v in ke.items()}},
+           "kron": {"ms": ms_k, "kernel_ms": kk[0] / steps, "nnz_K": K.nvals, "rows_K": K.nrows,
+                    "alg_bytes": alg_k, "GB/s": alg_k / (kk[0] / steps * 1e-3) / 1e9,
+                    "frac": alg_k / (kk[0] / steps * 1e-3) / 1e9 / peak_gbs},
+           "gpu_launches": state["launches"], "step_ms": state["step_ms"]}
+    for M in (A, B, E, G, R, K):
+        M.free()
+    return out
+
+
+def aux_closure(sp, steps, warmup):
+    """configs[3]: transitive closure C += C.C to the fixed point of the
+    2^18-vertex edge-labelled DAG (label-0 + label-1 union)."""
+    timed, state = aux_timer(sp, steps, warmup)
+    n = 1 << 18
+    (a0, b0), (a1, b1) = spgen.labeled_dag(n, 0.25, seed=9, device="cuda")
+    L0 = sp.Matrix.from_pairs(n, n, a0, b0)
+    L1 = sp.Matrix.from_pairs(n, n, a1, b1)
+    U = sp.ewise_add(L0, L1)
+    L0.free()
+    L1.free()
+    st = {}
+
+    def step():
+        C = U.duplicate()
+        st["it"] = sp.TransitiveClosure(C)
+        st["nnz"] = C.nvals
+        C.free()
+    ms_c = timed(step)
+    kt = {k: sp.kernel_timing(k)[0] / steps for k in AUX_GROUPS}
+    sp.set_kernel_timing(False)
+    out = {"ms": ms_c, "unit": "ms", "vertices": n, "nnz_in": U.nvals, "nnz_closure": st["nnz"],
+           "iterations": st["it"], "ms_per_iteration": ms_c / st["it"], "kernel_ms_per_step": kt,
+           "kernel_ms_total": sum(kt.values()), "gpu_launches": state["launches"], "step_ms": state["step_ms"]}
+    U.free()
+    return out
+
+
+def run_aux(args):
+    """--workload ewise_kron | closure18: the configs[2] / configs[3] rows on
+    their own JSON line (they are also embedded in the default line under
+    "aux").  1 GPU (replicas-only at N > 1)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import paper_conf_ipps_orachevkkg21_b200 as sp
+    torch.cuda.set_device(0)
+    sp.Initialize(0)
+    peak_gbs, peak_src = load_peaks()
+    steps, warmup = args.steps, max(args.warmup, 3)
     clocks = ClockSampler(0)
     if args.workload == "ewise_kron":
-        n = 1 << 20
-        r1, c1 = spgen.rmat_pairs(20, 16, 0.45, 0.22, 0.22, seed=1, device="cuda")
-        r2, c2 = spgen.uniform_pairs(n, n, 8, seed=2, device="cuda")
-        A = sp.Matrix.from_pairs(n, n, r1, c1)
-        B = sp.Matrix.from_pairs(n, n, r2, c2)
-        E = sp.Matrix.new(n, n)
-        ms_e = timed(lambda: sp.Matrix_EWiseAdd(E, A, B))
-        ke = {k: sp.kernel_timing(k) for k in ("ewise_split", "ewise_merge")}
-        sp.set_kernel_timing(False)
-        # algorithmic bytes: both inputs read once (colidx + rowptr), output written once
-        alg_e = 4 * (A.nvals + B.nvals) + 16 * (n + 1) + 4 * E.nvals + 8 * (n + 1)
-        rg, cg = spgen.rmat_pairs(10, 16, 0.45, 0.22, 0.22, seed=3, device="cuda")
-        rr, cr = spgen.rsm_pairs(64, 1, 2, seed=4, device="cuda")
-        G = sp.Matrix.from_pairs(1024, 1024, rg, cg)
-        R = sp.Matrix.from_pairs(64, 64, rr, cr)
-        K = sp.Matrix.new(1024 * 64, 1024 * 64)
-        ms_k = timed(lambda: sp.Kronecker(K, G, R))
-        kk = sp.kernel_timing("kron")
-        sp.set_kernel_timing(False)
-        alg_k = 4 * K.nvals + 8 * (K.nrows + 1)  # output-write bound (inputs are KB)
-        clk = clocks.stop()
-        per_e = (ke["ewise_split"][0] + ke["ewise_merge"][0]) / steps
+        r = aux_ewise_kron(sp, steps, warmup, peak_gbs)
         line = {"metric": "configs[2] EWiseAdd (2^20 rows) + Kronecker (2^10 x 64-state RSM): ms, GB/s vs HBM peak",
-                "value": ms_e + ms_k, "unit": "ms", "higher_is_better": False, "n_gpus": 1, "steps": steps,
-                "warmup": warmup, "dtype": "u32", "data": "synthetic (DESIGN.md §3)",
-                "config": {"workload": "ewise_kron", "baseline_config": "configs[2]",
-                           "l2": "256 MB write between timed steps"},
-                "ewise": {"ms": ms_e, "kernel_ms": per_e, "nnz_A": A.nvals, "nnz_B": B.nvals, "nnz_C": E.nvals,
-                          "alg_bytes": alg_e, "GB/s": alg_e / (per_e * 1e-3) / 1e9,
-                          "frac": alg_e / (per_e * 1e-3) / 1e9 / peak_gbs,
-                          "kernel_ms_per_step": {k: v[0] / steps for k, v in ke.items()}},
-                "kron": {"ms": ms_k, "kernel_ms": kk[0] / steps, "nnz_K": K.nvals, "rows_K": K.nrows,
-                         "alg_bytes": alg_k, "GB/s": alg_k / (kk[0] / steps * 1e-3) / 1e9,
-                         "frac": alg_k / (kk[0] / steps * 1e-3) / 1e9 / peak_gbs},
-                "peak": peak_gbs, "peak_source": peak_src, "clocks": clk}
+                "value": r["ms"], "config": {"workload": "ewise_kron", "baseline_config": "configs[2]",
+                                             "l2": "256 MB write between timed steps"},
+                "ewise": r["ewise"], "kron": r["kron"], "peak": peak_gbs, "peak_source": peak_src}
     else:
-        n = 1 << 18
-        (a0, b0), (a1, b1) = spgen.labeled_dag(n, 0.25, seed=9, device="cuda")
-        L0 = sp.Matrix.from_pairs(n, n, a0, b0)
-        L1 = sp.Matrix.from_pairs(n, n, a1, b1)
-        U = sp.ewise_add(L0, L1)
-        state = {}
-
-        def step():
-            C = U.duplicate()
-            state["it"] = sp.TransitiveClosure(C)
-            state["nnz"] = C.nvals
-            C.free()
-        ms_c = timed(step)
-        groups = ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "dense_ovf", "compact")
-        kt = {k: sp.kernel_timing(k)[0] / steps for k in groups}
-        sp.set_kernel_timing(False)
-        clk = clocks.stop()
+        r = aux_closure(sp, steps, warmup)
         line = {"metric": "configs[3] transitive closure C += C.C to fixed point (2^18-vertex labelled DAG): ms",
-                "value": ms_c, "unit": "ms", "higher_is_better": False, "n_gpus": 1, "steps": steps,
-                "warmup": warmup, "dtype": "u32", "data": "synthetic (DESIGN.md §3)",
-                "config": {"workload": "closure18", "baseline_config": "configs[3]", "vertices": n,
-                           "nnz_in": U.nvals, "nnz_closure": state["nnz"], "iterations": state["it"],
-                           "l2": "256 MB write between timed steps"},
-                "ms_per_iteration": ms_c / state["it"], "kernel_ms_per_step": kt, "clocks": clk}
-    line["gpu_launches"] = sum(launches)
-    line["step_ms"] = step_lists
-    line["value_is"] = "median of the timed steps (each step list in step_ms)"
+                "value": r["ms"], "config": {"workload": "closure18", "baseline_config": "configs[3]",
+                                             "vertices": r["vertices"], "nnz_in": r["nnz_in"],
+                                             "nnz_closure": r["nnz_closure"], "iterations": r["iterations"],
+                                             "l2": "256 MB write between timed steps"},
+                "ms_per_iteration": r["ms_per_iteration"], "kernel_ms_per_step": r["kernel_ms_per_step"]}
+    line.update({"unit": "ms", "higher_is_better": False, "n_gpus": 1, "steps": steps, "warmup": warmup,
+                 "dtype": "u32", "data": "synthetic (DESIGN.md §3)", "clocks": clocks.stop(),
+                 "gpu_launches": r["gpu_launches"], "step_ms": r["step_ms"],
+                 "value_is": "median of the timed steps (each step list in step_ms)"})
     print(json.dumps(line), flush=True)
 
 
@@ -317,6 +359,7 @@ def main():
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-aux", action="store_true", help="skip the configs[2]/[3] rows in the default line")
     args = ap.parse_args()
     if args.workload in AUX_WORKLOADS:
         return run_aux(args)
@@ -520,11 +563,23 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rp_h, ci_h = A.to_csr()
-        p, dt, nr_s, k, _ = cpu_oracle_sample(rp_h, ci_h, ub.cpu().numpy(),
-                                              float(os.environ.get("CPU_SAMPLE_PRODUCTS", "8e7")))
-        cpu = {"value": p / dt / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"every {k}-th row ({nr_s} rows, {p} products) of {args.workload}; "
-                         f"{dt:.1f}s single-threaded std::set Gustavson"}
+        p, dt, nr_s, thr, _ = cpu_oracle_sample(rp_h, ci_h, ub.cpu().numpy(),
+                                                float(os.environ.get("CPU_SAMPLE_PRODUCTS", "2e8")))
+        cpu = {"value": p / dt / 1e9, "unit": UNIT, "cores": thr, "kind": "oracle",
+               "sample": f"{4 * thr} contiguous row chunks spread over {args.workload} ({nr_s} rows, {p} products); "
+                         f"{dt:.1f}s wall of the unchanged std::set Gustavson oracle on {thr} threads"}
+
+    # ---- the other BASELINE rows (configs[2], configs[3]), 1 GPU ----------------
+    aux = None
+    if world == 1 and not args.no_aux:
+        C.free()
+        A.free()
+        torch.cuda.empty_cache()
+        aux_steps, aux_warm = max(args.steps, 9), 5
+        aux = {"configs[2] ewise_kron": aux_ewise_kron(sp, aux_steps, aux_warm, peak_gbs),
+               "configs[3] closure18": aux_closure(sp, aux_steps, aux_warm),
+               "note": "device-timed medians (CUDA events on the library stream, 256 MB L2 flush per step); "
+                       "step lists in step_ms"}
 
     if rank == 0:
         a_, b_, c_ = wl["abc"] if wl["abc"] else (None, None, None)
@@ -544,6 +599,7 @@ def main():
             "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": e2e,
+            "aux": aux,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

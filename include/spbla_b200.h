@@ -69,7 +69,12 @@ typedef enum {
     SPBLA_HINT_ACCUMULATE = 1u << 1,    /* MxM: C += A x B instead of C = A x B */
     SPBLA_HINT_SORTED = 1u << 2,        /* Build: pairs sorted by (row, col) ... */
     SPBLA_HINT_NO_DUPLICATES = 1u << 3, /* ... and duplicate-free: skip the sort */
-    SPBLA_HINT_VALIDATE = 1u << 4       /* Import/Wrap: check the CSR invariants */
+    SPBLA_HINT_VALIDATE = 1u << 4,      /* Import/Wrap: check the CSR invariants */
+    SPBLA_HINT_CLOSURE_STEP = 1u << 5   /* MxM with ACCUMULATE: a closure step C += C x C (or a
+                                           row shard of one); rows whose products exceed 4x
+                                           their current length skip the hash bins (mostly
+                                           repeated columns) -- a scheduling hint, the result
+                                           is the same */
 } spbla_Hint;
 
 /* ---- library state --------------------------------------------------- */

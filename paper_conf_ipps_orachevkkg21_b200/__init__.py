@@ -16,8 +16,8 @@ import ctypes
 import numpy as np
 
 from . import _capi
-from ._capi import (HINT_ACCUMULATE, HINT_HOST_MEMORY, HINT_NO, HINT_NO_DUPLICATES,  # noqa: F401
-                    HINT_SORTED, HINT_VALIDATE)
+from ._capi import (HINT_ACCUMULATE, HINT_CLOSURE_STEP, HINT_HOST_MEMORY, HINT_NO,  # noqa: F401
+                    HINT_NO_DUPLICATES, HINT_SORTED, HINT_VALIDATE)
 
 __all__ = [
     "SpblaError", "Initialize", "Finalize", "SetStream", "Synchronize", "memory_stats",
@@ -346,9 +346,11 @@ def Matrix_ExtractPairs(m: Matrix, device: bool = False):
     return m.extract_pairs(device)
 
 
-def MxM(C: Matrix, A: Matrix, B: Matrix, accumulate: bool = False):
-    """C = A x B, or C += A x B."""
-    _check(_lib().spbla_MxM(C.handle, A.handle, B.handle, HINT_ACCUMULATE if accumulate else 0), "spbla_MxM")
+def MxM(C: Matrix, A: Matrix, B: Matrix, accumulate: bool = False, closure_step: bool = False):
+    """C = A x B, or C += A x B; closure_step (with
+    accumulate): scheduling hint for a closure step C += C x C."""
+    hints = (HINT_ACCUMULATE if accumulate else 0) | (HINT_CLOSURE_STEP if closure_step else 0)
+    _check(_lib().spbla_MxM(C.handle, A.handle, B.handle, hints), "spbla_MxM")
 
 
 def Matrix_EWiseAdd(C: Matrix, A: Matrix, B: Matrix):

@@ -60,6 +60,7 @@ HINT_ACCUMULATE = 1 << 1
 HINT_SORTED = 1 << 2
 HINT_NO_DUPLICATES = 1 << 3
 HINT_VALIDATE = 1 << 4
+HINT_CLOSURE_STEP = 1 << 5
 
 STATUS_NAMES = {
     0: "SUCCESS", 1: "ERROR", 2: "DEVICE_ERROR", 3: "INVALID_ARGUMENT", 4: "INVALID_STATE",

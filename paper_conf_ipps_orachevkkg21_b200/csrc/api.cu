@@ -7,7 +7,7 @@
 #include <string>
 
 namespace spbla {
-void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate);
+void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate, uint32_t dup_ratio = 0);
 int transitive_closure(Matrix* C);
 void ewise_add(Matrix* C, const Matrix* A, const Matrix* B);
 void kronecker(Matrix* K, const Matrix* A, const Matrix* B);
@@ -324,7 +324,7 @@ spbla_Status spbla_MxM(spbla_Matrix C, spbla_Matrix A, spbla_Matrix B, uint32_t 
     return guarded([&] {
         require_init();
         NEED(C && A && B, "null matrix");
-        mxm(C, A, B, (hints & SPBLA_HINT_ACCUMULATE) != 0);
+        mxm(C, A, B, (hints & SPBLA_HINT_ACCUMULATE) != 0, (hints & SPBLA_HINT_CLOSURE_STEP) ? 4u : 0u);
     });
 }
 

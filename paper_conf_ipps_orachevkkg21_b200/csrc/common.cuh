@@ -53,6 +53,8 @@ void dev_free(void* p, size_t bytes);
 // read `n` uint64 words from device memory (synchronises the stream)
 void trace_mark(const char* what);
 void read_words(const uint64_t* dev, uint64_t* host, int n);
+// wait for the library stream by polling (no thread sleep; see context.cu)
+void stream_sync_spin();
 // read_words plus up to 128 more bytes from dev2 into host2, one synchronisation
 void read_words2(const uint64_t* dev, uint64_t* host, int n, const void* dev2, void* host2, size_t bytes2);
 void memset_async(void* p, int v, size_t bytes);
@@ -152,6 +154,9 @@ struct SegSource {
 #define SPBLA_WARP_MAX 256
 #endif
 constexpr uint64_t kRangeMinUb = SPBLA_WARP_MAX;
+// Bit 63 of a row's ub: the producer expects the row to be duplicate-heavy
+// (closure steps: products >> the row's current length); the engine masks it.
+constexpr uint64_t kUbDupFlag = uint64_t(1) << 63;
 void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, const uint2* range,
                 Matrix* out);
 

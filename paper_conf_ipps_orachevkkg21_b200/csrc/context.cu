@@ -91,10 +91,34 @@ void trace_mark(const char* what) {
     last = now;
 }
 
+// Wait for the library stream by polling an event instead of
+// cudaStreamSynchronize: the runtime's default (blocking/yield) wait puts the
+// host thread to sleep at every size read-back, and on the GPU boxes the
+// wake-up costs 0.1-1 ms and occasionally tens of ms (measured on the configs[3]
+// closure, 12 read-backs per step: 16 voluntary context switches per step,
+// 8-15 ms medians with 40-230 ms outliers; tools/stall_probe.py).  The read-backs
+// are short waits on a GPU that is about to finish, so spinning is the cheap
+// choice.
+void stream_sync_spin() {
+    static cudaEvent_t ev = nullptr;
+    static int dev = -1;
+    if (dev != g_ctx.device) {
+        if (ev) cudaEventDestroy(ev);
+        CUDA_CHECK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        dev = g_ctx.device;
+    }
+    CUDA_CHECK(cudaEventRecord(ev, g_ctx.stream));
+    for (;;) {
+        const cudaError_t e = cudaEventQuery(ev);
+        if (e == cudaSuccess) return;
+        if (e != cudaErrorNotReady) CUDA_CHECK(e);
+    }
+}
+
 void read_words(const uint64_t* dev, uint64_t* host, int n) {
     CUDA_CHECK(cudaMemcpyAsync(g_ctx.host_words, dev, n * sizeof(uint64_t), cudaMemcpyDeviceToHost,
                                g_ctx.stream));
-    CUDA_CHECK(cudaStreamSynchronize(g_ctx.stream));
+    stream_sync_spin();
     std::memcpy(host, g_ctx.host_words, n * sizeof(uint64_t));
 }
 
@@ -103,7 +127,7 @@ void read_words2(const uint64_t* dev, uint64_t* host, int n, const void* dev2, v
     unsigned char* hw = reinterpret_cast<unsigned char*>(g_ctx.host_words);
     CUDA_CHECK(cudaMemcpyAsync(hw, dev, n * sizeof(uint64_t), cudaMemcpyDeviceToHost, g_ctx.stream));
     CUDA_CHECK(cudaMemcpyAsync(hw + 128, dev2, bytes2, cudaMemcpyDeviceToHost, g_ctx.stream));
-    CUDA_CHECK(cudaStreamSynchronize(g_ctx.stream));
+    stream_sync_spin();
     std::memcpy(host, hw, n * sizeof(uint64_t));
     std::memcpy(host2, hw + 128, bytes2);
 }
@@ -179,6 +203,13 @@ void ktime_end(int slot) {
 }
 
 void ktime_enable(bool on) {
+    // events are created up front: a cudaEventCreate inside a timed step
+    // showed up as a slow first timed step
+    while (on && g_kevpool.size() < 8192) {
+        cudaEvent_t e;
+        CUDA_CHECK(cudaEventCreate(&e));
+        g_kevpool.push_back(e);
+    }
     g_ktime_on = on;
     g_krec.clear();
     g_kev_used = 0;

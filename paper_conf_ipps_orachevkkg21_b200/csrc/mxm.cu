@@ -41,7 +41,7 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
                               const uint2* __restrict__ bspan, const uint4* __restrict__ binfo,
                               const off_t64* __restrict__ crp,
                               const idx_t* __restrict__ cci, uint64_t* __restrict__ ub, uint2* __restrict__ range,
-                              uint4* __restrict__ desc, uint32_t* __restrict__ nseg) {
+                              uint4* __restrict__ desc, uint32_t* __restrict__ nseg, uint32_t dup_ratio) {
     const unsigned lane = threadIdx.x & 31, g = lane & (kGroup - 1);
     const unsigned gshift = lane & ~(kGroup - 1);  // first lane of this row's group
     const size_t ngroups = (size_t(gridDim.x) * blockDim.x) / kGroup;
@@ -53,6 +53,7 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
         uint64_t s = 0;
         off_t64 b = 0, e = 0;
         uint32_t cn = 0, cl = 0;  // running non-empty count / product prefix of the row
+        uint32_t lcr = 0;         // |C[r]| (accumulate)
         idx_t lo = 0xFFFFFFFFu, hi = 0;
         uint4* drow = nullptr;
         if (valid) {
@@ -72,6 +73,7 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
                     }
                     cn = 1;
                     cl = lc;
+                    lcr = lc;
                 }
             }
         }
@@ -119,7 +121,10 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
             hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, d, kGroup));
         }
         if (valid && g == 0) {
-            ub[r] = s;
+            // dup_ratio (closure steps): products far above the row's current
+            // length mean mostly repeated columns (C[k] largely inside C[r])
+            const bool dup = dup_ratio && s > kRangeMinUb && s > uint64_t(dup_ratio) * lcr;
+            ub[r] = s | (dup ? kUbDupFlag : 0);
             nseg[r] = cn;
             if (s > kRangeMinUb) range[r] = make_uint2(lo, hi);
         }
@@ -128,7 +133,7 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
 
 }  // namespace
 
-static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
+static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate, uint32_t dup_ratio) {
     if (A->ncols != B->nrows || C->nrows != A->nrows || C->ncols != B->ncols)
         SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "MxM: shapes do not conform");
     if (!C->owned) SPBLA_THROW(SPBLA_STATUS_INVALID_ARGUMENT, "MxM: output matrix is a non-owning view");
@@ -161,11 +166,11 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     if (info)
         mxm_ub_kernel<true><<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, nullptr, binfo.p, crp,
                                                             accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p,
-                                                            nseg.p);
+                                                            nseg.p, dup_ratio);
     else
         mxm_ub_kernel<false><<<grid, 256, 0, ctx().stream>>>(view(A), B->rowptr, B->colidx, bspan.p, nullptr, crp,
                                                              accumulate ? C->colidx : nullptr, ub.p, range.p, desc.p,
-                                                             nseg.p);
+                                                             nseg.p, dup_ratio);
     ktime_end(tk);
     count_launch();
     check_launch("mxm_ub_kernel");
@@ -186,9 +191,9 @@ static void mxm_impl(Matrix* C, const Matrix* A, const Matrix* B, bool accumulat
     trace_mark("mxm done");
 }
 
-void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
+void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate, uint32_t dup_ratio) {
     try {
-        mxm_impl(C, A, B, accumulate);
+        mxm_impl(C, A, B, accumulate, accumulate ? dup_ratio : 0u);
     } catch (...) {
         // a non-accumulating MxM may have released C already: leave it a
         // valid empty matrix rather than a dangling one
@@ -202,12 +207,16 @@ void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate) {
     }
 }
 
+constexpr uint32_t kClosureDupRatio = 4;
+
 int transitive_closure(Matrix* C) {
     if (C->nrows != C->ncols) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "closure: matrix must be square");
     int it = 0;
     uint64_t prev = C->nnz;
     for (;;) {
-        mxm(C, C, C, true);
+        // closure steps: rows whose products exceed kClosureDupRatio x their
+        // current length are routed to the bitmap kernel
+        mxm(C, C, C, true, kClosureDupRatio);
         ++it;
         if (C->nnz == prev) break;  // C only grows: equal nnz <=> fixed point
         prev = C->nnz;

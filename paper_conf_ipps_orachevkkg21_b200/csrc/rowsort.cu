@@ -64,10 +64,11 @@ __shared__ unsigned long long s_probe_ext[12];
 #define PROBE(i) do {} while (0)
 #define PROBE_PRINT(tag, u, ns) do {} while (0)
 #endif
-constexpr int kNumBins = 13;
+constexpr int kNumBins = 14;
 enum {
     BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_H0,
-    BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_H6, BIN_DENSE = 12
+    BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_H6, BIN_DENSE = 12,
+    BIN_DUP = 13  // rows flagged duplicate-heavy (kUbDupFlag): straight to the small bitmap kernel
 };
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 // hash bins: ub limits (each sized so its tables fit the residency below)
@@ -1041,17 +1042,23 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
 }
 
 // ---- 1. binning ------------------------------------------------------------
-__global__ void bin_count_kernel(const uint64_t* __restrict__ ub, idx_t nrows, idx_t ncols,
-                                 uint64_t* __restrict__ cap, uint8_t* __restrict__ bin,
+__global__ void bin_count_kernel(const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t nrows,
+                                 idx_t ncols, uint64_t* __restrict__ cap, uint8_t* __restrict__ bin,
                                  uint32_t* __restrict__ counts, uint32_t* __restrict__ hist) {
     __shared__ uint32_t sh[kNumBins];
     if (threadIdx.x < kNumBins) sh[threadIdx.x] = 0;
     __syncthreads();
     for (size_t r = blockIdx.x * size_t(blockDim.x) + threadIdx.x; r < nrows;
          r += size_t(gridDim.x) * blockDim.x) {
-        uint64_t u = ub[r];
+        const uint64_t uf = ub[r], u = uf & ~kUbDupFlag;
         cap[r] = u < ncols ? u : uint64_t(ncols);
         int b = bin_of(u);
+        // a duplicate-heavy row (flagged by the producer) whose span fits two
+        // small bitmap windows skips the hash bins: its duplicates would
+        // overflow the 16-slot buckets and send it to the same bitmap kernel
+        // after a wasted gather
+        if ((uf & kUbDupFlag) && b >= BIN_H0 && b <= BIN_H6 && range && range[r].y - range[r].x < kSmallSpan)
+            b = BIN_DUP;
         bin[r] = uint8_t(b);
         if (b == BIN_EMPTY) counts[r] = 0;
         atomicAdd(&sh[b], 1u);
@@ -1105,7 +1112,7 @@ __global__ void make_recs_kernel(SegSource src, const idx_t* __restrict__ rows, 
         const idx_t r = rows[i];
         RowRec x;
         x.r = r;
-        x.u = uint32_t(min(ub[r], uint64_t(0xFFFFFFFFu)));
+        x.u = uint32_t(min(ub[r] & ~kUbDupFlag, uint64_t(0xFFFFFFFFu)));
         if (range) {
             const uint2 rg = range[r];
             x.clo = rg.x;
@@ -1505,21 +1512,22 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    // meta: hist[13] binoff[14] cursor[13] work[9] ovf[4] work2[1]
+    // meta: hist[14] binoff[15] cursor[14] work[9] ovf[4] work2[1] work3[1]
     DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
-    uint32_t* binoff = meta.p + 13;
-    uint32_t* cursor = meta.p + 27;
-    uint32_t* work = meta.p + 40;
-    uint32_t* ovf = meta.p + 49;  // fallback lists: [0, ovf[1]) and [nrows, ovf[3])
-    uint32_t* work2 = meta.p + 53;
+    uint32_t* binoff = meta.p + 14;
+    uint32_t* cursor = meta.p + 29;
+    uint32_t* work = meta.p + 43;
+    uint32_t* ovf = meta.p + 52;  // fallback lists: [0, ovf[1]) and [nrows, ovf[3])
+    uint32_t* work2 = meta.p + 56;
+    uint32_t* work3 = meta.p + 57;
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
     {
         const uint32_t lst1[2] = {nrows, nrows};
         copy_async(ovf + 2, lst1, sizeof(lst1), cudaMemcpyHostToDevice);
     }
     const unsigned gb = (unsigned)std::min<uint64_t>(ceil_div(nrows, 256), uint64_t(nsm) * 8);
-    bin_count_kernel<<<gb, 256, 0, st>>>(ub, nrows, ncols, cap.p, bin.p, counts.p, hist);
+    bin_count_kernel<<<gb, 256, 0, st>>>(ub, range, nrows, ncols, cap.p, bin.p, counts.p, hist);
     count_launch();
     check_launch("bin_count_kernel");
     exclusive_scan_u64(cap.p, soff.p, nrows);
@@ -1558,6 +1566,13 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     if (hcnt[BIN_DENSE]) {
         DENSE<<<grid_for(BIN_DENSE, nsm), 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols,
                                                               scratch.p, soff.p, counts.p, work);
+        count_launch();
+    }
+    ktime_end(t);
+    t = ktime_begin("dense_ovf", st);
+    if (hcnt[BIN_DUP]) {  // duplicate-heavy rows flagged by the producer
+        SDENSE<<<std::min<uint32_t>(nsm * kSDPerSM, hcnt[BIN_DUP]), 256, kSDSmem, st>>>(
+            src, rows.p, binoff + BIN_DUP, range, ncols, scratch.p, soff.p, counts.p, work3);
         count_launch();
     }
     ktime_end(t);

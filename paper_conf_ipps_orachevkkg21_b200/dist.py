@@ -87,10 +87,10 @@ class CudaOps:
         B.assemble_row_blocks(blocks)
         return B
 
-    def mxm(self, C, A, B, accumulate):
+    def mxm(self, C, A, B, accumulate, closure_step=False):
         if C is None:
             C = self.sp.Matrix.new(A.nrows, B.ncols)
-        self.sp.MxM(C, A, B, accumulate=accumulate)
+        self.sp.MxM(C, A, B, accumulate=accumulate, closure_step=closure_step)
         return C
 
 
@@ -124,7 +124,7 @@ def distributed_closure(ops, C_local, n, group=None, max_iters=10_000):
     it = 0
     while it < max_iters:
         B = gather_rows(ops, C_local, n, n, group)
-        C_local = ops.mxm(C_local, C_local, B, True)
+        C_local = ops.mxm(C_local, C_local, B, True, closure_step=True)
         it += 1
         cur = allreduce_int(ops.nvals(C_local), group, device=dev)
         if cur == prev:

@@ -33,7 +33,7 @@ class OracleOps:
         assert len(rp) == nrows + 1
         return oracle.Csr(nrows, ncols, rp, np.concatenate(cis) if cis else np.zeros(0, np.uint32))
 
-    def mxm(self, C, A, B, accumulate):
+    def mxm(self, C, A, B, accumulate, closure_step=False):
         return oracle.mxm(A, B, C if accumulate else None)
 
 

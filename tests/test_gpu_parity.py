@@ -306,6 +306,26 @@ def test_closure_labeled_dag(sp):
     assert it == oit
 
 
+def test_mxm_closure_step_hint_dup_rows(sp):
+    """SPBLA_HINT_CLOSURE_STEP routes rows with products > 4x their length
+    (duplicate-heavy) to the bitmap kernel: C += C.C on a partly closed DAG
+    (hash-bin-sized dup-heavy rows), bit-exact vs the oracle, with and
+    without the hint."""
+    n = 1 << 14
+    (r0, c0), (r1, c1) = spgen.labeled_dag(n, 0.6, seed=83)
+    r = np.concatenate([r0.numpy(), r1.numpy()])
+    c = np.concatenate([c0.numpy(), c1.numpy()])
+    C, OC = both_from_pairs(sp, n, n, r, c)
+    for step in range(5):
+        want = oracle.mxm(OC, OC, OC)
+        D = C.duplicate()
+        sp.MxM(C, C, C, accumulate=True, closure_step=True)
+        sp.MxM(D, D, D, accumulate=True)
+        assert_same(C, want, f"C += C.C with the hint, step {step}")
+        assert_same(D, want, f"C += C.C without the hint, step {step}")
+        OC = want
+
+
 def test_closure_rmat_small(sp):
     r, c = spgen.rmat_pairs(9, 2, 0.45, 0.22, 0.22, seed=81)
     A, OA = both_from_pairs(sp, 512, 512, r, c)
