@@ -157,6 +157,14 @@ spbla_Status spbla_Matrix_Wrap(spbla_Matrix* matrix, spbla_Index nrows, spbla_In
 /* Borrow the device pointers of a matrix (valid until it is modified/freed). */
 spbla_Status spbla_Matrix_DevicePointers(spbla_Matrix matrix, const spbla_Offset** rowptr,
                                          const spbla_Index** colidx);
+/* Write `matrix` as one row block of a larger CSR matrix (PAPER.md l.253-257
+ * storage; DESIGN.md §7 row partitioning): rowptr[i] = matrix.rowptr[i] +
+ * offset for i in [0, nrows] (nrows + 1 entries) and colidx[0, nvals) =
+ * matrix.colidx -- device arrays owned by the caller (typically the shard's
+ * slice of an all-gather buffer), asynchronous on the library stream.
+ * Errors: null matrix / rowptr, null colidx for a non-empty matrix. */
+spbla_Status spbla_Matrix_ExportRowBlock(spbla_Matrix matrix, spbla_Offset* rowptr, spbla_Index* colidx,
+                                        spbla_Offset offset);
 /* Concatenate row blocks (block b: nrows[b] rows, device arrays rowptr[b]
  * starting at 0 and colidx[b] with nnz[b] values) into `matrix` (replaced;
  * its ncols is kept; sum nrows[b] must equal its nrows).  Used to assemble a

@@ -315,6 +315,14 @@ class Matrix:
                else torch.empty(0, dtype=torch.int32, device=dev))
         return trp, tci
 
+    def export_row_block(self, rowptr, colidx, offset: int):
+        """Write this matrix as one row block of a larger CSR matrix into the
+        device tensors rowptr (int64, nrows+1: entries + offset) and colidx
+        (int32, nvals)."""
+        n = self.nvals
+        _check(_lib().spbla_Matrix_ExportRowBlock(self._h, rowptr.data_ptr(), colidx.data_ptr() if n else None,
+                                                  int(offset)), "spbla_Matrix_ExportRowBlock")
+
     def assemble_row_blocks(self, blocks):
         """Replace content by the concatenation of row blocks
         [(nrows_b, rowptr_b tensor, colidx_b tensor, nnz_b), ...] (device)."""

@@ -17,6 +17,7 @@ void submatrix(Matrix* R, const Matrix* M, idx_t i0, idx_t j0, idx_t nr, idx_t n
 void matrix_build(Matrix* m, const idx_t* rows, const idx_t* cols, uint64_t n, uint32_t hints);
 void matrix_extract_pairs(const Matrix* m, idx_t* rows, idx_t* cols, uint32_t hints);
 void matrix_export(const Matrix* m, off_t64* rowptr, idx_t* colidx, uint32_t hints);
+void matrix_export_block(const Matrix* m, off_t64* rowptr_out, idx_t* colidx_out, off_t64 offset);
 void matrix_import(Matrix* m, const off_t64* rowptr, const idx_t* colidx, uint64_t nnz, uint32_t hints);
 void matrix_duplicate(const Matrix* m, Matrix* d);
 void matrix_assemble(Matrix* m, uint32_t nblocks, const idx_t* nrows, const off_t64* const* rowptr,
@@ -269,6 +270,16 @@ spbla_Status spbla_Matrix_ExportCSR(spbla_Matrix m, spbla_Offset* rowptr, spbla_
         NEED(m, "null matrix");
         NEED(m->nnz == 0 || colidx || !rowptr, "null colidx buffer");
         matrix_export(m, rowptr, colidx, hints);
+    });
+}
+
+spbla_Status spbla_Matrix_ExportRowBlock(spbla_Matrix m, spbla_Offset* rowptr, spbla_Index* colidx,
+                                        spbla_Offset offset) {
+    return guarded([&] {
+        require_init();
+        NEED(m && rowptr, "null argument");
+        NEED(m->nnz == 0 || colidx, "null colidx buffer");
+        matrix_export_block(m, rowptr, colidx, offset);
     });
 }
 

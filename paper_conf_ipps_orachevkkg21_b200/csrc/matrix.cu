@@ -205,6 +205,19 @@ void matrix_duplicate(const Matrix* m, Matrix* d) {
     matrix_import(d, m->rowptr, m->colidx, m->nnz, 0);
 }
 
+// Export m as one row block of a larger matrix: rowptr_out[i] = rowptr[i] +
+// offset for i in [0, nrows] (nrows + 1 entries), colidx_out = colidx (device
+// arrays, stream-ordered, no synchronisation).  The all-gather of a
+// row-partitioned matrix writes every shard straight into its slice of the
+// gathered buffers with this.
+void matrix_export_block(const Matrix* m, off_t64* rowptr_out, idx_t* colidx_out, off_t64 offset) {
+    shift_rowptr_kernel<<<grid_for(uint64_t(m->nrows) + 1, 256), 256, 0, ctx().stream>>>(m->rowptr, m->nrows + 1,
+                                                                                       offset, rowptr_out);
+    count_launch();
+    check_launch("shift_rowptr_kernel");
+    if (m->nnz) copy_async(colidx_out, m->colidx, m->nnz * sizeof(idx_t), cudaMemcpyDeviceToDevice);
+}
+
 void matrix_assemble(Matrix* m, uint32_t nblocks, const idx_t* nrows, const off_t64* const* rowptr,
                      const idx_t* const* colidx, const uint64_t* nnz) {
     if (!m->owned) SPBLA_THROW(SPBLA_STATUS_INVALID_ARGUMENT, "Assemble: matrix is a non-owning view");

@@ -8,8 +8,7 @@ transitive closure all-gathers the new C shards every iteration and tests the
 fixed point with an all-reduce of nnz.
 
 The local operations go through an ``ops`` object so the host-side protocol
-(partitioning, padded all-gather of variable-size CSR blocks, fixed-point
-loop) is exercised by world_size-2 gloo tests on CPU with the oracle as the
+(partitioning, exact-size all-gather of CSR row blocks, fixed-point loop) is exercised by world_size-2 gloo tests on CPU with the oracle as the
 local multiply; production uses :class:`CudaOps` (the CUDA library).
 """
 from __future__ import annotations
@@ -35,39 +34,48 @@ def product_balanced_bounds(row_weight: torch.Tensor, world: int):
     return bounds
 
 
-def allgather_csr(rowptr: torch.Tensor, colidx: torch.Tensor, group=None):
-    """All-gather variable-size CSR row blocks.  ``rowptr`` (int64, starts at
-    0, nrows+1) and ``colidx`` (int32) of this rank's block; returns
-    [(nrows_b, rowptr_b, colidx_b, nnz_b)] for every rank in rank order.
-    Blocks are padded to the largest one for the collective."""
+def allgather_rows(ops, M_local, nrows_total, ncols, group=None):
+    """All-gather a row-partitioned matrix (every rank's block of rows, in
+    rank order) into ONE CSR: the block sizes are exchanged first, every rank
+    writes its own block straight into its slice of the gathered rowptr /
+    colidx buffers (offsets shifted on the device by ``ops.export_block``),
+    and one broadcast per rank fills the other slices -- exact sizes, no
+    padding and no second copy.  Returns the gathered matrix (``ops.wrap``)."""
     world = dist.get_world_size(group)
-    dev = rowptr.device
-    if dev.type == "cuda" and dist.get_backend(group) == "gloo":
-        # gloo path (CPU tests / single-GPU multi-rank runs): collective on host copies
-        blocks = allgather_csr(rowptr.cpu(), colidx.cpu(), group)
-        return [(nr, rp.to(dev), ci.to(dev), nz) for nr, rp, ci, nz in blocks]
-    nrows = rowptr.numel() - 1
-    nnz = colidx.numel()
-    sizes = torch.tensor([nrows, nnz], dtype=torch.int64, device=dev)
-    all_sizes = torch.empty(world * 2, dtype=torch.int64, device=dev)
-    dist.all_gather_into_tensor(all_sizes, sizes, group=group)
-    all_sizes = all_sizes.view(world, 2).cpu().tolist()
-    max_rows = max(s[0] for s in all_sizes)
-    max_nnz = max(max(s[1] for s in all_sizes), 1)
-    rp = torch.zeros(max_rows + 1, dtype=torch.int64, device=dev)
-    rp[:nrows + 1] = rowptr
-    ci = torch.zeros(max_nnz, dtype=torch.int32, device=dev)
-    ci[:nnz] = colidx
-    rp_all = torch.empty(world * (max_rows + 1), dtype=torch.int64, device=dev)
-    ci_all = torch.empty(world * max_nnz, dtype=torch.int32, device=dev)
-    dist.all_gather_into_tensor(rp_all, rp, group=group)
-    dist.all_gather_into_tensor(ci_all, ci, group=group)
-    out = []
+    rank = dist.get_rank(group)
+    nrows, nnz = ops.shape_nnz(M_local)
+    dev = ops.device(M_local)
+    gloo = dist.get_backend(group) == "gloo"
+    sdev = "cpu" if gloo else dev
+    sizes = torch.tensor([nrows, nnz], dtype=torch.int64, device=sdev)
+    all_sizes = [torch.empty_like(sizes) for _ in range(world)]
+    dist.all_gather(all_sizes, sizes, group=group)
+    all_sizes = [tuple(int(v) for v in t.cpu()) for t in all_sizes]
+    assert sum(s[0] for s in all_sizes) == nrows_total, "row blocks do not cover the matrix"
+    total = sum(s[1] for s in all_sizes)
+    rbase = [0] * world
+    nbase = [0] * world
+    for b in range(1, world):
+        rbase[b] = rbase[b - 1] + all_sizes[b - 1][0]
+        nbase[b] = nbase[b - 1] + all_sizes[b - 1][1]
+    rp_all = torch.empty(nrows_total + 1, dtype=torch.int64, device=dev)
+    ci_all = torch.empty(max(total, 1), dtype=torch.int32, device=dev)
+    ops.export_block(M_local, rp_all[rbase[rank]:rbase[rank] + nrows + 1], ci_all[nbase[rank]:nbase[rank] + nnz],
+                     nbase[rank])
     for b, (nr, nz) in enumerate(all_sizes):
-        rpb = rp_all[b * (max_rows + 1): b * (max_rows + 1) + nr + 1]
-        cib = ci_all[b * max_nnz: b * max_nnz + nz]
-        out.append((nr, rpb, cib, nz))
-    return out
+        # (block b's first offset equals block b-1's last: overlapping
+        # slices receive identical values)
+        for t in (rp_all[rbase[b]:rbase[b] + nr + 1], ci_all[nbase[b]:nbase[b] + nz]):
+            if t.numel() == 0:
+                continue
+            if gloo and t.device.type != "cpu":  # gloo (CPU tests, one-GPU multi-rank runs): via host
+                h = t.cpu()
+                dist.broadcast(h, src=b, group=group)
+                if b != rank:
+                    t.copy_(h)
+            else:
+                dist.broadcast(t, src=b, group=group)
+    return ops.wrap(nrows_total, ncols, rp_all, ci_all, total)
 
 
 class CudaOps:
@@ -76,16 +84,20 @@ class CudaOps:
     def __init__(self, sp):
         self.sp = sp
 
-    def csr(self, M):
-        return M.device_tensors()
+    def shape_nnz(self, M):
+        return M.nrows, M.nvals
+
+    def device(self, M):
+        return M.device_tensors()[0].device
 
     def nvals(self, M):
         return M.nvals
 
-    def assemble(self, blocks, nrows, ncols):
-        B = self.sp.Matrix.new(nrows, ncols)
-        B.assemble_row_blocks(blocks)
-        return B
+    def export_block(self, M, rowptr, colidx, offset):
+        M.export_row_block(rowptr, colidx, offset)
+
+    def wrap(self, nrows, ncols, rowptr, colidx, nnz):
+        return self.sp.Matrix.wrap(nrows, ncols, rowptr, colidx, nvals=nnz)
 
     def mxm(self, C, A, B, accumulate, closure_step=False):
         if C is None:
@@ -103,9 +115,7 @@ def allreduce_int(x: int, group=None, op=dist.ReduceOp.SUM, device=None) -> int:
 
 
 def gather_rows(ops, M_local, nrows_total, ncols, group=None):
-    rp, ci = ops.csr(M_local)
-    blocks = allgather_csr(rp, ci, group)
-    return ops.assemble(blocks, nrows_total, ncols)
+    return allgather_rows(ops, M_local, nrows_total, ncols, group)
 
 
 def distributed_mxm(ops, A_local, B_local, nrows_B, ncols_B, group=None, C_local=None, accumulate=False):
@@ -119,7 +129,7 @@ def distributed_closure(ops, C_local, n, group=None, max_iters=10_000):
     """C += C x C to the fixed point with C row-partitioned: every iteration
     all-gathers the C shards (B = C), updates the local rows, and all-reduces
     nnz to detect the fixed point.  Returns (C_local, iterations)."""
-    dev = ops.csr(C_local)[0].device
+    dev = ops.device(C_local)
     prev = allreduce_int(ops.nvals(C_local), group, device=dev)
     it = 0
     while it < max_iters:

@@ -1,7 +1,8 @@
 """Row-partitioned multi-GPU protocol (dist.py) on CPU: world_size 2, gloo,
-the oracle as the local multiply.  Checks that partitioning + padded
-all-gather of CSR blocks + assembly reproduce the single-process results of
-MxM and of the closure loop (rows, nnz and iteration count)."""
+the oracle as the local multiply.  Checks that partitioning + the exact-size
+all-gather of CSR row blocks (each rank writes its block into its slice, one
+broadcast per rank) reproduce the single-process results of MxM and of the
+closure loop (rows, nnz and iteration count)."""
 import os
 import socket
 
@@ -17,21 +18,25 @@ from paper_conf_ipps_orachevkkg21_b200 import dist as spdist
 
 
 class OracleOps:
-    def csr(self, M):
-        return (torch.as_tensor(M.rowptr.astype(np.int64)), torch.as_tensor(M.colidx.astype(np.int32)))
+    """The dist.py ops on CPU tensors with the oracle as the local multiply."""
+
+    def shape_nnz(self, M):
+        return M.nrows, M.nvals
+
+    def device(self, M):
+        return torch.device("cpu")
 
     def nvals(self, M):
         return M.nvals
 
-    def assemble(self, blocks, nrows, ncols):
-        rps, cis, base = [np.zeros(1, np.uint64)], [], 0
-        for nr, rp, ci, nz in blocks:
-            rps.append(rp[1:].numpy().astype(np.uint64) + np.uint64(base))
-            cis.append(ci.numpy().astype(np.uint32))
-            base += nz
-        rp = np.concatenate(rps)
-        assert len(rp) == nrows + 1
-        return oracle.Csr(nrows, ncols, rp, np.concatenate(cis) if cis else np.zeros(0, np.uint32))
+    def export_block(self, M, rowptr, colidx, offset):
+        rowptr.copy_(torch.as_tensor(M.rowptr.astype(np.int64) + offset))
+        if M.nvals:
+            colidx.copy_(torch.as_tensor(M.colidx.astype(np.int64)).to(torch.int32))
+
+    def wrap(self, nrows, ncols, rowptr, colidx, nnz):
+        return oracle.Csr(nrows, ncols, rowptr.numpy().astype(np.uint64),
+                          colidx[:nnz].numpy().astype(np.uint32))
 
     def mxm(self, C, A, B, accumulate, closure_step=False):
         return oracle.mxm(A, B, C if accumulate else None)
