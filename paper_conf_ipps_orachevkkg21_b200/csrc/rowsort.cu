@@ -916,7 +916,8 @@ template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS, bool FCOUNT>
 __global__ void __launch_bounds__(THREADS)
 dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
                  const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
-                 const uint64_t* __restrict__ soff, uint32_t* __restrict__ counts, uint32_t* __restrict__ work) {
+                 const uint64_t* __restrict__ soff, const uint64_t* __restrict__ ub, uint32_t* __restrict__ counts,
+                 uint32_t* __restrict__ work) {
     constexpr int NW = THREADS / 32;
     constexpr uint32_t kWords = BITS / 32, kTop = kWords / 32;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -964,9 +965,47 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         const uint32_t nwin = uint32_t((span + BITS - 1) / BITS);
         idx_t* out = scratch + soff[r];
         uint32_t written = 0;
+        // Partition mode (a span of more than three windows, e.g. a heavy row
+        // over 2^26 columns): instead of one gather per window, count the
+        // products per window (gather 1), scatter them by window into the
+        // row's own output region (gather 2; its capacity holds every product
+        // when ub <= ncols), then each window reads only its slice.  The
+        // window-w emission writes below the start of slice w+1 (distinct <=
+        // products), so it never overwrites an unread slice.  Two gathers
+        // and a slice pass per row, whatever the number of windows.
+        const uint64_t prods = ub[r] & ~kUbDupFlag;
+        const bool part = nwin > 3 && prods <= soff[r + 1] - soff[r] && nwin < 2 * BATCH;
+        uint32_t* wcur = bm;               // (partition mode, during the gathers) per-window cursors
+        uint32_t* wbeg = bm + kWords / 2;  // ... and slice starts (nwin + 1 entries)
+        uint32_t* slb = reinterpret_cast<uint32_t*>(sd_ptr);  // slice bounds while the windows run
+        if (part) {
+            for (uint32_t i = threadIdx.x; i < nwin; i += THREADS) wcur[i] = 0u;
+            __syncthreads();
+            block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH,
+                                           false, [&](idx_t c) { atomicAdd(&wcur[(c - clo) / BITS], 1u); });
+            if (threadIdx.x == 0) {  // exclusive scan of < 2*BATCH window counts (rare rows: serial is fine)
+                uint32_t acc = 0;
+                for (uint32_t i = 0; i < nwin; ++i) {
+                    const uint32_t v = wcur[i];
+                    wbeg[i] = acc;
+                    wcur[i] = acc;
+                    acc += v;
+                }
+                wbeg[nwin] = acc;
+            }
+            __syncthreads();
+            block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH,
+                                           false, [&](idx_t c) { out[atomicAdd(&wcur[(c - clo) / BITS], 1u)] = c; });
+            // (the barrier ending the gather orders the scatter before the slice reads)
+            for (uint32_t i = threadIdx.x; i <= nwin; i += THREADS) slb[i] = wbeg[i];  // descriptors are dead now
+            __syncthreads();
+            for (uint32_t i = threadIdx.x; i < kWords; i += THREADS) bm[i] = 0u;  // the counters lived in the bitmap
+            __syncthreads();
+        }
         for (uint32_t w = 0; w < nwin; ++w) {
             const uint64_t wlo = uint64_t(clo) + uint64_t(w) * BITS;
             const uint64_t whi = min(wlo + BITS, uint64_t(chi) + 1);
+            const uint32_t sb = part ? slb[w] : 0u, se = part ? slb[w + 1] : 0u;  // this window's slice of out
             // the window's used top words are split evenly over the warps
             // (a fixed split left the warps outside the row's span idle)
             const uint32_t used = uint32_t((whi - wlo + 1023) >> 10);
@@ -976,8 +1015,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
             // the gather (s_w is clean before the gather's staging barrier),
             // so the emission needs one walk instead of two
             if (FCOUNT && threadIdx.x < NW) s_w[threadIdx.x] = 0u;
-            block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH, false,
-                                           [&](idx_t c) {
+            auto set_bit = [&](idx_t c) {
                 if (c >= wlo && c < whi) {
                     const uint32_t d = uint32_t(c - wlo);
                     const uint32_t bit = 1u << (d & 31);
@@ -985,7 +1023,15 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                     if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
                     if (FCOUNT && !(old & bit)) atomicAdd(&s_w[(d >> 10) / tcw], 1u);
                 }
-            });
+            };
+            if (part) {  // this window's slice: coalesced reads of the scattered products
+                if (FCOUNT) __syncthreads();  // (the s_w clear before any count)
+                for (uint32_t i = sb + threadIdx.x; i < se; i += THREADS) set_bit(out[i]);
+                __syncthreads();
+            } else {
+                block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH,
+                                               false, set_bit);
+            }
             // emission over the top level: warp w owns top words [tb, te),
             // read 32 at a time (one per lane); a ballot gives the non-zero
             // ones and the warp visits only those (rows of a few hundred
@@ -1565,14 +1611,14 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     t = ktime_begin("dense", st);
     if (hcnt[BIN_DENSE]) {
         DENSE<<<grid_for(BIN_DENSE, nsm), 1024, kDSmem, st>>>(src, rows.p, binoff + BIN_DENSE, range, ncols,
-                                                              scratch.p, soff.p, counts.p, work);
+                                                              scratch.p, soff.p, ub, counts.p, work);
         count_launch();
     }
     ktime_end(t);
     t = ktime_begin("dense_ovf", st);
     if (hcnt[BIN_DUP]) {  // duplicate-heavy rows flagged by the producer
         SDENSE<<<std::min<uint32_t>(nsm * kSDPerSM, hcnt[BIN_DUP]), 256, kSDSmem, st>>>(
-            src, rows.p, binoff + BIN_DUP, range, ncols, scratch.p, soff.p, counts.p, work3);
+            src, rows.p, binoff + BIN_DUP, range, ncols, scratch.p, soff.p, ub, counts.p, work3);
         count_launch();
     }
     ktime_end(t);
@@ -1601,9 +1647,9 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     t = ktime_begin("dense_ovf", st);
     if (hash_rows) {  // (fallback rows come only from the hash bins)
         const uint32_t g = std::min<uint32_t>(nsm * kSDPerSM, hash_rows);
-        SDENSE<<<g, 256, kSDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, counts.p, work2);
+        SDENSE<<<g, 256, kSDSmem, st>>>(src, ovf_rows.p, ovf, range, ncols, scratch.p, soff.p, ub, counts.p, work2);
         DENSE<<<std::min<uint32_t>(nsm, hash_rows), 1024, kDSmem, st>>>(src, ovf_rows.p, ovf + 2, range, ncols,
-                                                                        scratch.p, soff.p, counts.p, work + 6);
+                                                                        scratch.p, soff.p, ub, counts.p, work + 6);
         count_launch(2);
     }
     ktime_end(t);

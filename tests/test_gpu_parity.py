@@ -345,3 +345,28 @@ def test_generator_cpu_gpu_identical():
     (a, b), (x, y) = spgen.labeled_dag(5000, 0.25, seed=4)
     (a2, b2), (x2, y2) = spgen.labeled_dag(5000, 0.25, seed=4, device="cuda")
     assert torch.equal(b, b2.cpu()) and torch.equal(y, y2.cpu())
+
+
+def test_mxm_heavy_rows_wide_span_partition(sp):
+    """Heavy rows (> 40960 products, the dense bin) over ncols = 2^26: 43
+    bitmap windows, handled by the partition-by-window mode (two gathers and
+    one slice pass per row instead of one gather per window); also a
+    small-span heavy row and a wide heavy row with duplicate columns."""
+    ncols = 1 << 26
+    rng = np.random.default_rng(37)
+    k = 300
+    rb = np.repeat(np.arange(k), 500).astype(np.uint32)                     # B: 300 rows x ~500 entries
+    cb = rng.integers(0, ncols, len(rb)).astype(np.uint32)
+    cb[: 500 * 10] = rng.integers(0, 5000, 500 * 10).astype(np.uint32)      # rows 0..9: narrow columns
+    ra = np.concatenate([np.repeat(np.arange(4), 150),                       # 4 heavy wide rows (~75K products)
+                         np.full(10, 4),                                     # narrow-span heavy-ish row
+                         rng.integers(5, 40, 400)]).astype(np.uint32)
+    ca = np.concatenate([rng.integers(10, k, 600), np.arange(10),
+                         rng.integers(0, k, 400)]).astype(np.uint32)
+    # B rows 100..109 are copies of row 100 and row 0 uses all of them:
+    # duplicate columns across its segments
+    cb.reshape(k, 500)[101:110] = cb.reshape(k, 500)[100]
+    ca[:10] = np.arange(100, 110)
+    A, OA = both_from_pairs(sp, 40, k, ra, ca)
+    B, OB = both_from_pairs(sp, k, ncols, rb, cb)
+    assert_same(sp.mxm(A, B), oracle.mxm(OA, OB), "heavy rows over 2^26 columns")
