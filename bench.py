@@ -221,12 +221,13 @@ def aux_timer(sp, steps, warmup):
     state = {"launches": 0, "step_ms": []}
 
     def timed(fn):
+        # timed steps without the per-kernel event records (a host-launched
+        # loop of ~100 small launches per step would carry their cost); one
+        # extra step afterwards records the kernel breakdown
         for i in range(warmup):
-            if i == warmup - 1:
-                sp.set_kernel_timing(True)
             fn()
         torch.cuda.synchronize()
-        sp.set_kernel_timing(True)
+        sp.set_kernel_timing(False)
         sp.reset_launch_count()
         ms = []
         for _ in range(steps):
@@ -239,6 +240,9 @@ def aux_timer(sp, steps, warmup):
             e1.synchronize()
             ms.append(e0.elapsed_time(e1))
         state["launches"] += sp.launch_count()
+        sp.set_kernel_timing(True)
+        fn()  # (the kernel breakdown step: kernel_timing() reads its records, per step)
+        torch.cuda.synchronize()
         log(f"[aux] step ms: {[round(x, 2) for x in ms]}")
         state["step_ms"].append([round(x, 3) for x in ms])
         # median: these host-launched ops can see rare host stalls; the full
@@ -272,15 +276,15 @@ def aux_ewise_kron(sp, steps, warmup, peak_gbs):
     kk = sp.kernel_timing("kron")
     sp.set_kernel_timing(False)
     alg_k = 4 * K.nvals + 8 * (K.nrows + 1)  # output-write bound (inputs are KB)
-    per_e = (ke["ewise_split"][0] + ke["ewise_merge"][0]) / steps
+    per_e = ke["ewise_split"][0] + ke["ewise_merge"][0]  # (one breakdown step)
     out = {"ms": ms_e + ms_k, "unit": "ms",
            "ewise": {"ms": ms_e, "kernel_ms": per_e, "nnz_A": A.nvals, "nnz_B": B.nvals, "nnz_C": E.nvals,
                      "alg_bytes": alg_e, "GB/s": alg_e / (per_e * 1e-3) / 1e9,
                      "frac": alg_e / (per_e * 1e-3) / 1e9 / peak_gbs,
-                     "kernel_ms_per_step": {k: v[0] / steps for k, v in ke.items()}},
-           "kron": {"ms": ms_k, "kernel_ms": kk[0] / steps, "nnz_K": K.nvals, "rows_K": K.nrows,
-                    "alg_bytes": alg_k, "GB/s": alg_k / (kk[0] / steps * 1e-3) / 1e9,
-                    "frac": alg_k / (kk[0] / steps * 1e-3) / 1e9 / peak_gbs},
+                     "kernel_ms_per_step": {k: v[0] for k, v in ke.items()}},
+           "kron": {"ms": ms_k, "kernel_ms": kk[0], "nnz_K": K.nvals, "rows_K": K.nrows,
+                    "alg_bytes": alg_k, "GB/s": alg_k / (kk[0] * 1e-3) / 1e9,
+                    "frac": alg_k / (kk[0] * 1e-3) / 1e9 / peak_gbs},
            "gpu_launches": state["launches"], "step_ms": state["step_ms"]}
     for M in (A, B, E, G, R, K):
         M.free()
@@ -306,7 +310,7 @@ def aux_closure(sp, steps, warmup):
         st["nnz"] = C.nvals
         C.free()
     ms_c = timed(step)
-    kt = {k: sp.kernel_timing(k)[0] / steps for k in AUX_GROUPS}
+    kt = {k: sp.kernel_timing(k)[0] for k in AUX_GROUPS}  # (one breakdown step)
     sp.set_kernel_timing(False)
     out = {"ms": ms_c, "unit": "ms", "vertices": n, "nnz_in": U.nvals, "nnz_closure": st["nnz"],
            "iterations": st["it"], "ms_per_iteration": ms_c / st["it"], "kernel_ms_per_step": kt,

@@ -92,6 +92,7 @@ spbla_Status spbla_Finalize(void) {
     return guarded([&] {
         Context& c = ctx();
         if (c.device < 0) return;
+        release_cached_blocks();
         CUDA_CHECK(cudaStreamSynchronize(c.stream));
         cudaMemPoolTrimTo(c.pool, 0);
         if (c.mat_pool) cudaMemPoolDestroy(c.mat_pool);

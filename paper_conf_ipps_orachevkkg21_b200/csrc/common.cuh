@@ -50,6 +50,8 @@ void require_init();
 // with temporaries (a pool miss maps fresh memory: ~60 ms per GB on B200).
 void* dev_alloc(size_t bytes, bool mat = false);
 void dev_free(void* p, size_t bytes);
+// give the size-class cache's blocks back to the pools (Finalize, OOM retry)
+void release_cached_blocks();
 // read `n` uint64 words from device memory (synchronises the stream)
 void trace_mark(const char* what);
 void read_words(const uint64_t* dev, uint64_t* host, int n);

@@ -289,7 +289,9 @@ void ewise_add(Matrix* C, const Matrix* A, const Matrix* B) {
     DevBuf<uint64_t> ta(2 * (ntiles + 1));
     DevBuf<uint64_t> status(ntiles + 1);
     memset_async(status.p, 0, status.n * sizeof(uint64_t));
-    // the result: colidx capacity nnzA + nnzB (>= nnz(C)); the exact nnz is read back
+    // the result: colidx capacity nnzA + nnzB (>= nnz(C)); the exact nnz is
+    // read back, and a result with more than 1/8 of that capacity unused is
+    // moved into an exact-size buffer
     DevBuf<off_t64> rp(size_t(A->nrows) + 1, kMat);
     DevBuf<idx_t> ci(m.L, kMat);
     int t = ktime_begin("ewise_split", ctx().stream);
@@ -314,6 +316,15 @@ void ewise_add(Matrix* C, const Matrix* A, const Matrix* B) {
     uint64_t nnz;
     read_words(rp.p + A->nrows, &nnz, 1);
     size_t rc = rp.n, cc = ci.n;
+    if (m.L - nnz > m.L / 8) {
+        // many shared entries (e.g. A + A): keep an exact-size colidx instead
+        // of holding nnzA + nnzB words for the matrix's lifetime
+        DevBuf<idx_t> exact(nnz, kMat);
+        if (nnz) copy_async(exact.p, ci.p, nnz * sizeof(idx_t), cudaMemcpyDeviceToDevice);
+        cc = exact.n;
+        matrix_replace(C, rp.detach(), rc, exact.detach(), cc, nnz);
+        return;
+    }
     matrix_replace(C, rp.detach(), rc, ci.detach(), cc, nnz);
 }
 

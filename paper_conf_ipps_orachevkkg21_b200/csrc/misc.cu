@@ -67,7 +67,63 @@ __global__ void sub_copy_kernel(const idx_t* __restrict__ ci, const uint64_t* __
     }
 }
 
+// Set difference per row, D = C \ P (the semi-naive closure's new entries,
+// DESIGN.md §4.2): warp per row, every C entry binary-searched in P's row,
+// kept entries placed by ballot.  WRITE = false counts, true writes.
+template <bool WRITE>
+__global__ void row_diff_kernel(CsrView C, CsrView P, uint32_t* __restrict__ cnt, const off_t64* __restrict__ rp,
+                                idx_t* __restrict__ out) {
+    const unsigned lane = lane_id();
+    const size_t nw = size_t(gridDim.x) * (blockDim.x >> 5);
+    for (size_t r = (blockIdx.x * size_t(blockDim.x) + threadIdx.x) >> 5; r < C.nrows; r += nw) {
+        const off_t64 b = C.rowptr[r], e = C.rowptr[r + 1];
+        const off_t64 pb = P.rowptr[r], pe = P.rowptr[r + 1];
+        uint64_t o = WRITE ? rp[r] : 0;
+        for (off_t64 q0 = b; q0 < e; q0 += 32) {
+            const off_t64 q = q0 + lane;
+            bool keep = false;
+            idx_t c = 0;
+            if (q < e) {
+                c = C.colidx[q];
+                const uint64_t at = lb64(P.colidx, pb, pe, c);
+                keep = at == pe || P.colidx[at] != c;
+            }
+            const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+            if (WRITE && keep) out[o + __popc(bal & ((1u << lane) - 1u))] = c;
+            o += __popc(bal);
+        }
+        if (!WRITE && lane == 0) cnt[r] = uint32_t(o);
+    }
+}
+
 }  // namespace
+
+void row_difference(Matrix* D, const Matrix* C, const Matrix* P) {
+    if (C->nrows != P->nrows || C->ncols != P->ncols || D->nrows != C->nrows || D->ncols != C->ncols)
+        SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "difference: shapes differ");
+    const idx_t m = C->nrows;
+    if (m == 0 || C->nnz == 0) {
+        matrix_set_empty(D);
+        return;
+    }
+    DevBuf<uint32_t> cnt(m);
+    DevBuf<off_t64> rp(size_t(m) + 1, kMat);
+    const unsigned g = grid_for(uint64_t(m) * 32, 256);
+    row_diff_kernel<false><<<g, 256, 0, ctx().stream>>>(view(C), view(P), cnt.p, nullptr, nullptr);
+    count_launch();
+    check_launch("row_diff_kernel");
+    exclusive_scan_u32(cnt.p, rp.p, m);
+    uint64_t nnz;
+    read_words(rp.p + m, &nnz, 1);
+    DevBuf<idx_t> ci(nnz, kMat);
+    if (nnz) {
+        row_diff_kernel<true><<<g, 256, 0, ctx().stream>>>(view(C), view(P), nullptr, rp.p, ci.p);
+        count_launch();
+        check_launch("row_diff_kernel");
+    }
+    size_t rc = rp.n, cc = ci.n;
+    matrix_replace(D, rp.detach(), rc, ci.detach(), cc, nnz);
+}
 
 void transpose(Matrix* T, const Matrix* M) {
     if (T->nrows != M->ncols || T->ncols != M->nrows) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "Transpose: T must be n x m");

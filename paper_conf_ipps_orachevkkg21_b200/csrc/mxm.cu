@@ -209,17 +209,63 @@ void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate, uint32_t 
 
 constexpr uint32_t kClosureDupRatio = 4;
 
+void matrix_duplicate(const Matrix* m, Matrix* d);
+void row_difference(Matrix* D, const Matrix* C, const Matrix* P);
+
+namespace {
+struct OwnedMatrix {  // a library-internal matrix released on scope exit
+    Matrix m;
+    OwnedMatrix(idx_t r, idx_t c) {
+        m.nrows = r;
+        m.ncols = c;
+    }
+    ~OwnedMatrix() {
+        try {
+            matrix_release(&m);
+        } catch (...) {
+        }
+    }
+};
+void swap_storage(Matrix* a, Matrix* b) { std::swap(*a, *b); }
+}  // namespace
+
+// Transitive closure C += C x C to the fixed point (§I l.113-117,
+// l.126; R9).  Squaring step k: C_{k+1} = C_k + C_k C_k.  With
+// Delta_k = C_k \ C_{k-1} the same iterate is C_k + Delta_k C_k + C_k Delta_k
+// (C_{k-1} C_{k-1} is inside C_k already), the semi-naive step: two products
+// with the small Delta instead of one with C.  The loop switches to it when
+// the last step added less than 1/kSemiNaiveDiv of the entries (|Delta| is
+// known from the nnz read-backs), typically the final confirming step; the
+// iterates and the iteration count are those of the plain loop.
+constexpr uint64_t kSemiNaiveDiv = 8;
+
 int transitive_closure(Matrix* C) {
     if (C->nrows != C->ncols) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "closure: matrix must be square");
-    int it = 0;
-    uint64_t prev = C->nnz;
-    for (;;) {
-        // closure steps: rows whose products exceed kClosureDupRatio x their
-        // current length are routed to the bitmap kernel
-        mxm(C, C, C, true, kClosureDupRatio);
+    const idx_t n = C->nrows;
+    OwnedMatrix prev(n, n);  // C_{k-1}
+    matrix_duplicate(C, &prev.m);
+    // closure steps: rows whose products exceed kClosureDupRatio x their
+    // current length are routed to the bitmap kernel
+    mxm(C, C, C, true, kClosureDupRatio);
+    int it = 1;
+    while (C->nnz != prev.m.nnz) {  // C only grows: equal nnz <=> fixed point
+        const uint64_t added = C->nnz - prev.m.nnz;
+        if (added * kSemiNaiveDiv < C->nnz) {
+            OwnedMatrix delta(n, n);
+            row_difference(&delta.m, C, &prev.m);
+            OwnedMatrix next(n, n);
+            matrix_duplicate(C, &next.m);
+            mxm(&next.m, &delta.m, C, true, kClosureDupRatio);  // C + Delta C
+            mxm(&next.m, C, &delta.m, true, kClosureDupRatio);  // ... + C Delta
+            swap_storage(&prev.m, C);                           // prev = C_k
+            swap_storage(C, &next.m);                           // C = C_{k+1} (next holds the old prev)
+        } else {
+            matrix_release(&prev.m);
+            prev.m.nrows = prev.m.ncols = n;
+            matrix_duplicate(C, &prev.m);
+            mxm(C, C, C, true, kClosureDupRatio);
+        }
         ++it;
-        if (C->nnz == prev) break;  // C only grows: equal nnz <=> fixed point
-        prev = C->nnz;
     }
     return it;
 }

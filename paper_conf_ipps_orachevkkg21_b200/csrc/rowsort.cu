@@ -1396,39 +1396,53 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
             if (threadIdx.x == 0) s_beg[nr] = int32_t(kCT);
         }
         __syncthreads();
+        // thread-owned 4-word chunks c = k*kCThreads + tid of the tile: the
+        // destination is one aligned 16-B store; the chunk's 4 source words
+        // (one row's run, shifted by that row's slack, any alignment) are 4
+        // coalesced word loads.  The row check is per chunk, not per word.
+        constexpr int kCChunks = kCItems / 4;
         idx_t v[kCItems];
         if (staged) {
-            // element e = k*kCThreads + t of the tile; the row advances rarely
-            // (rows average thousands of elements), by binary search over the
-            // staged starts when it does
             uint32_t ri = 0;
             int32_t nxt = s_beg[1];
             const idx_t* sp = s_src[0];
 #pragma unroll
-            for (int k = 0; k < kCItems; ++k) {
-                const int32_t e = k * kCThreads + int32_t(threadIdx.x);
-                if (e >= nxt) {
-                    uint32_t lo = ri + 1, hi = nr - 1;  // last row with start <= e
-                    while (lo < hi) {
-                        const uint32_t mid = (lo + hi + 1) >> 1;
-                        if (s_beg[mid] <= e) lo = mid; else hi = mid - 1;
+            for (int k = 0; k < kCChunks; ++k) {
+                const int32_t e0 = 4 * (k * kCThreads + int32_t(threadIdx.x));
+                if (e0 + 3 < nxt) {  // the whole chunk in the current row (rows average thousands of words)
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        if (uint32_t(e0 + j) < n) v[4 * k + j] = sp[e0 + j];
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int32_t e = e0 + j;
+                        if (e >= nxt) {  // next row(s): binary search over the staged starts
+                            uint32_t lo = ri + 1, hi = nr - 1;  // last row with start <= e
+                            while (lo < hi) {
+                                const uint32_t mid = (lo + hi + 1) >> 1;
+                                if (s_beg[mid] <= e) lo = mid; else hi = mid - 1;
+                            }
+                            ri = lo;
+                            nxt = s_beg[ri + 1];
+                            sp = s_src[ri];
+                        }
+                        if (uint32_t(e) < n) v[4 * k + j] = sp[e];
                     }
-                    ri = lo;
-                    nxt = s_beg[ri + 1];
-                    sp = s_src[ri];
                 }
-                if (uint32_t(e) < n) v[k] = sp[e];
             }
         } else {
 #pragma unroll
-            for (int k = 0; k < kCItems; ++k) {
-                const uint32_t e = k * kCThreads + threadIdx.x;
-                if (e < n) {
-                    const uint64_t d = d0 + e;
-                    const uint32_t r = row_of(rowptr, r0, r1, d);
-                    v[k] = buf[d + (soff[r] - rowptr[r])];
+            for (int k = 0; k < kCChunks; ++k)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const uint32_t e = 4 * (k * kCThreads + threadIdx.x) + j;
+                    if (e < n) {
+                        const uint64_t d = d0 + e;
+                        const uint32_t r = row_of(rowptr, r0, r1, d);
+                        v[4 * k + j] = buf[d + (soff[r] - rowptr[r])];
+                    }
                 }
-            }
         }
         // publish "read done": the barrier orders every thread's loads before
         // thread 0's gpu-scope fence and release store
@@ -1441,10 +1455,18 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
         for (uint32_t j = s_w.x + threadIdx.x; j < s_w.y; j += kCThreads)
             while (ld_acquire_u32(&flags[j]) == 0) __nanosleep(64);
         __syncthreads();
-        idx_t* dp = buf + d0 + threadIdx.x;
+        idx_t* dp = buf + d0;  // 16-B aligned (kCT and the buffer are)
 #pragma unroll
-        for (int k = 0; k < kCItems; ++k)
-            if (k * kCThreads + threadIdx.x < n) dp[k * kCThreads] = v[k];
+        for (int k = 0; k < kCChunks; ++k) {
+            const uint32_t e0 = 4 * (k * kCThreads + threadIdx.x);
+            if (e0 + 4 <= n) {
+                *reinterpret_cast<uint4*>(dp + e0) = make_uint4(v[4 * k], v[4 * k + 1], v[4 * k + 2], v[4 * k + 3]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    if (e0 + j < n) dp[e0 + j] = v[4 * k + j];
+            }
+        }
         __syncthreads();  // s_beg / s_t reuse
     }
 }
