@@ -107,12 +107,16 @@ void spbla_ResetLaunchCount(void);
 /* Per-kernel CUDA-event timing on each kernel's launching stream (bench.py's
  * roofline evidence).  enable != 0 clears previous records and starts
  * recording; spbla_GetKernelTiming sums the recorded launches of the named
- * kernel group ("mxm_ub", "warp_bins", "H1".."H6", "dense", "compact") and
- * synchronises on their end events. */
+ * kernel group and synchronises on their end events.  Groups: "mxm_ub"
+ * (B-row records + upper-bound pass), "warp_bins" (W1..W8), "H0".."H6"
+ * (block hash bins), "dense" (bitmap bin of the heaviest rows), "dense_ovf"
+ * (small bitmap kernel: duplicate-heavy and fallen-back rows), "compact",
+ * "ewise_split", "ewise_merge", "kron". */
 spbla_Status spbla_SetKernelTiming(int enable);
 spbla_Status spbla_GetKernelTiming(const char* name, double* total_ms, uint64_t* launches);
-/* Upper-bound ("ub") limits of the row engine's bins, ascending: warp bins
- * E=1,2,4,8,16, hash bins H1..H6; rows above the last go to the bitmap bin.  *n: capacity in, count out. */
+/* Upper-bound ("ub") limits of the row engine's bins, ascending (11 values):
+ * warp bins W1, W2, W4, W8 (32 E products), hash bins H0..H6; rows above the
+ * last go to the bitmap ("dense") bin.  *n: capacity in, count out. */
 spbla_Status spbla_GetEngineThresholds(uint64_t* thresholds, uint32_t* n);
 
 /* ---- matrix life cycle --------------------------- */

@@ -8,26 +8,23 @@
 // Pipeline (all on the device; two host read-backs for allocation sizes):
 //   1. bin_count   : cap[r] = min(ub[r], ncols), bin[r] by ub, bin histogram
 //   2. scan(cap)   : scratch offsets (in-house decoupled look-back scan)
-//   3. bin_scatter : row lists per bin
-//   4. per-bin kernels:
-//        warp bitonic (ub <= 32*E, E = 1..16): flattened gather into smem,
-//            register bitonic sort, shuffle dedup
-//        block hash (ub <= 2048 / 8192 / 24576, 256 / 512 / 1024 threads):
-//            a smem bitmap when the row's column span fits the table, else
-//            an ORDER-PRESERVING hash (home slot monotone in the column,
-//            linear probing upward, no wrap-around): clusters are mutually
-//            ordered, so emission writes each element at (#occupied slots
-//            before its cluster) + (rank inside the cluster) - sorted output
-//            without a sort; rows whose probes run long go to the bitmap bin
-//        block bitmap (heavier rows): two-level smem bitmap over the row's
-//            column span in windows of 2^20 bits; the top level (one bit per
-//            word) makes clearing and emission proportional to touched words
-//      block kernels stage compacted segment descriptors in smem (pointer
-//      pre-offset by the segment's concatenated start, inclusive end), then
-//      each warp walks 256 consecutive products: 32 candidate segments per
-//      lane-window, shuffle binary search, 8 independent loads in flight.
+//   3. bin_scatter : row lists per bin; make_recs: 40-B work records of the
+//                    hash-bin rows
+//   4. per-bin kernels (heaviest first, persistent grids):
+//        dense (ub > 40960): two-level smem bitmap over 1.5 Mi-column
+//            windows, one 1024-thread block per row; a span of more than
+//            three windows is partitioned by window first (two gathers)
+//        dense_ovf: the same kernel with 256 Ki-column windows for rows the
+//            producer flagged duplicate-heavy (closure steps) and for
+//            hash-bin rows that fell back
+//        hash H6..H0 (ub <= 40960 .. 512): bucketed order-preserving hash in
+//            smem (bucket = floor((c - lo) / W), 16 slots of 16-bit offsets,
+//            one atomicAdd per insert), 16x2 SIMD Batcher sort per bucket
+//            pair, warp-cooperative emission; a smem span bitmap when the
+//            span is small
+//        warp W8..W1 (ub <= 256): one warp per row, register bitonic sort
 //   5. scan(counts): CSR row offsets
-//   6. compact     : scratch -> colidx
+//   6. compact     : in-place move from capacity offsets to CSR offsets
 #include "common.cuh"
 
 #include <algorithm>
@@ -1742,7 +1739,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
 }
 
 void engine_thresholds(uint64_t* out, uint32_t* n) {
-    // ub upper limits of bins W1, W2, W4, W8, W16, H1..H6 (DENSE above)
+    // ub upper limits of bins W1, W2, W4, W8, H0..H6 (DENSE above)
     const uint64_t t[11] = {32, 64, 128, kWarpMaxUb, kH0, kH1, kH2, kH3, kH4, kH5, kH6};
     const uint32_t k = *n < 11 ? *n : 11;
     for (uint32_t i = 0; i < k; ++i) out[i] = t[i];
