@@ -28,6 +28,7 @@
 #include "common.cuh"
 
 #include <algorithm>
+#include <cuda/atomic>
 #include <cstdlib>
 
 namespace spbla {
@@ -216,7 +217,11 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
         for (uint32_t q0 = threadIdx.x * U; q0 < total; q0 += THREADS * U) {
             // a row already bound for the fallback stops gathering (per
             // thread: no barrier inside this loop)
-            if (abort && *abort) break;
+            // (a relaxed atomic load -- an ordinary LDS -- : the flag is set
+            // concurrently, by atomicExch, from inserting threads)
+            if (abort && cuda::atomic_ref<uint32_t, cuda::thread_scope_block>(*const_cast<uint32_t*>(abort))
+                             .load(cuda::memory_order_relaxed))
+                break;
             uint32_t k;
             if ((KINDT >= 0 ? KINDT : s.kind) == 1) {
                 k = 0;
@@ -270,6 +275,14 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
 template <int NW>
 __device__ __forceinline__ void scan_warp_counts(uint32_t* s_w) {
     const unsigned lane = lane_id();
+    if (NW == 1) {  // one warp: no scan (and no speculative reads of s_w[lane])
+        if (threadIdx.x == 0) {
+            s_w[32] = s_w[0];
+            s_w[0] = 0u;
+        }
+        __syncthreads();
+        return;
+    }
     if ((threadIdx.x >> 5) == 0) {
         const uint32_t v = lane < NW ? s_w[lane] : 0u;
         const uint32_t inc = warp_inclusive_scan(v);
@@ -496,10 +509,10 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     __shared__ uint32_t s_w[33];
     __shared__ uint32_t s_wt[KP][NW];
     // s_flag / s_novf are written (and s_flag read) during the gather, which
-    // starts without a barrier: they alternate by row parity, and row i
-    // clears row i+1's pair (row i-1's last reads precede the barrier that
-    // ended row i-1)
-    __shared__ uint32_t s_flag2[2], s_novf2[2], s_nob, s_pool;
+    // starts without a barrier: thread 0 clears them for the next row just
+    // before the barrier that ends the current row, after their last reads
+    // (the fallback decision, behind the pass-A / overflow barriers)
+    __shared__ uint32_t s_flag, s_novf, s_nob, s_pool;
     // early stop of the gather once the row is bound for the fallback: the
     // small bins, where duplicate-heavy closure rows overflow
     constexpr bool kEarlyStop = THREADS <= 128;
@@ -539,8 +552,8 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
 #pragma unroll 1
     for (uint32_t i = threadIdx.x; i < MAXB; i += THREADS) bcnt[i] = 0u;
     if (threadIdx.x == 0) {
-        s_flag2[0] = s_flag2[1] = 0;
-        s_novf2[0] = s_novf2[1] = 0;
+        s_flag = 0;
+        s_novf = 0;
     }
     // prologue: claim rows 0 and 1, plan row 0, stage its first batch
     // the pipeline thread is the last one: it has the least pass-A work
@@ -570,17 +583,17 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             have_nx = nxt1 < hi_i;
             if (have_nx) nx = recs[nxt1];
         }
-        // row-parity pair in every bin: the gather may start before thread 0
-        // reaches this point, so a row never clears its own flag/counter
-        const uint32_t fcur = it & 1u, fnext = (it + 1) & 1u;
-        uint32_t& s_flag = s_flag2[fcur];
-        uint32_t& s_novf = s_novf2[fcur];
-        if (threadIdx.x == 0) {
-            s_flag2[fnext] = 0;
-            s_novf2[fnext] = 0;
+        if (threadIdx.x == 0) {  // (used only behind this row's insert barrier)
             s_nob = 0;
             s_pool = 0;
         }
+        // the next row's gather starts right after this row's last barrier
+        auto clear_row_flags = [&]() {
+            if (threadIdx.x == 0) {
+                s_flag = 0;
+                s_novf = 0;
+            }
+        };
         // thread PT: plan of row i+1 into s_plan (visible after the next barrier)
         auto publish_next = [&]() {
             if (threadIdx.x == PT) {
@@ -610,6 +623,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             for (uint32_t i = threadIdx.x; i < nw; i += THREADS) bmw[i] = i < TABW ? 0xFFFFFFFFu : 0u;
             const RowPlan N = s_plan[(it + 1) & 1];
             pf_issue(N);
+            clear_row_flags();
             pf_commit(N);
             __syncthreads();
             continue;
@@ -621,6 +635,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             __syncthreads();
             const RowPlan N = s_plan[(it + 1) & 1];
             pf_issue(N);
+            clear_row_flags();
             pf_commit(N);
             __syncthreads();
             continue;
@@ -636,7 +651,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                 tab16[slot * (2 * MPP) + b] = uint16_t(d - b * W);
             } else {
                 const uint32_t i = atomicAdd(&s_novf, 1u);
-                if (i < OVCAP) ovl[i] = c; else s_flag = 1;
+                if (i < OVCAP) ovl[i] = c; else atomicExch(&s_flag, 1u);  // (polled concurrently: atomic)
             }
         }, kEarlyStop ? &s_flag : nullptr);
         PROBE(4);
@@ -816,19 +831,18 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                 const uint32_t jn = min(32u, np - mb);
 #pragma unroll 1
                 for (uint32_t j = 0; j < jn; j += 8) {
-                    // past the last pair a lane group repeats pair mb+j read-only:
-                    // it neither stores columns nor restores table words (the
-                    // owning group g4 = 0 restores them; no intra-warp
-                    // read/write overlap)
-                    const bool ok = j + g4 < jn;
-                    const uint32_t m = mb + j + (ok ? g4 : 0u);
+                    // past the row's last pair (np <= m < mb + 32 <= MP: MP and mb
+                    // are multiples of 32) a lane group works on a pair this row
+                    // never touched: its words are empty and its counters zero,
+                    // so it emits nothing and rewrites clean values that no
+                    // other lane reads (no aliasing of a live pair)
+                    const uint32_t m = mb + j + g4;
                     uint32_t* wp = tabw + (4 * t8) * MPP + m;
                     uint32_t wv[4];
 #pragma unroll
                     for (int k = 0; k < 4; ++k) wv[k] = wp[k * MPP];
 #pragma unroll
-                    for (int k = 0; k < 4; ++k)
-                        if (ok) wp[k * MPP] = 0xFFFFFFFFu;
+                    for (int k = 0; k < 4; ++k) wp[k * MPP] = 0xFFFFFFFFu;
                     uint32_t inc[4], ex;
                     if (DEDUP_B) {
                         uint32_t prevw = __shfl_up_sync(FULL, wv[3], 1, 4);
@@ -854,6 +868,8 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                         for (int k = 0; k < 4; ++k) inc[k] = uint32_t(k) * 0x00010001u;
                         ex = 4 * t8 * 0x00010001u;
                     }
+                    // (for a pair past np: zero counters, a stale offset, and every
+                    // store predicated off)
                     const uint2 nn = reinterpret_cast<const uint2*>(bcnt)[m];
                     const uint32_t pm = poff[m];
                     const uint32_t c0 = (nn.x & kOvfFlag) ? obcnt[nn.x & ~kOvfFlag] >> 16 : nn.x;
@@ -862,11 +878,12 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                     idx_t* o1 = out + (pm + c0 + (ex >> 16));
 #pragma unroll
                     for (int k = 0; k < 4; ++k)
-                        st_if(o0 + (inc[k] & 0xFFFFu), base0 + (wv[k] & 0xFFFFu), ok && (wv[k] & 0xFFFFu) != 0xFFFFu);
+                        st_if(o0 + (inc[k] & 0xFFFFu), base0 + (wv[k] & 0xFFFFu), (wv[k] & 0xFFFFu) != 0xFFFFu);
 #pragma unroll
                     for (int k = 0; k < 4; ++k)
-                        st_if(o1 + (inc[k] >> 16), base1 + (wv[k] >> 16), ok && (wv[k] >> 16) != 0xFFFFu);
-                    if (ok && t8 == 0) {
+                        st_if(o1 + (inc[k] >> 16), base1 + (wv[k] >> 16), (wv[k] >> 16) != 0xFFFFu);
+                    __syncwarp();  // the group's lanes have read the pair's counters
+                    if (t8 == 0) {
                         if ((nn.x | nn.y) & kOvfFlag) {  // overflowed bucket: its sorted extras follow the slots
                             if (nn.x & kOvfFlag) {
                                 const uint32_t e = obcnt[nn.x & ~kOvfFlag], mc = e >> 16, off = e & 0xFFFFu;
@@ -881,6 +898,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
                     }
                 }
             }
+            clear_row_flags();
             pf_commit(N);
             __syncthreads();
             PROBE(7);
@@ -888,6 +906,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             continue;
         }
         // ---- fallback: restore the pairs this row dirtied (each thread its own) --
+        __syncthreads();  // (every thread is past its reads of the row's flags)
         // (pass A touched only owned pairs; inserts and the overflow pass
         // touched pairs < np, all of which have an owner)
 #pragma unroll 1
@@ -896,6 +915,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             for (int sl = 0; sl < 16; ++sl) tabw[sl * MPP + m] = 0xFFFFFFFFu;
             reinterpret_cast<uint2*>(bcnt)[m] = make_uint2(0u, 0u);
         }
+        clear_row_flags();
         pf_commit(N);
         __syncthreads();
     }
