@@ -1303,8 +1303,15 @@ __global__ void compact_kernel(const idx_t* __restrict__ scratch, const uint64_t
 // point at lower tickets, held by running blocks that never wait before
 // publishing, so the chain cannot deadlock.  Tiles with zero slack are
 // already in place and only publish.
-constexpr int kCThreads = 256, kCItems = 32;
-constexpr uint32_t kCT = kCThreads * kCItems;  // 8192 elements per tile
+#ifndef SPBLA_CT_T  // threads, words per thread, blocks per SM (overridable for a sweep)
+// (configs[4] sweep, round 2: 128x32x8 14.08 ms < 96x32x10 14.25 < 128x24x10
+// 14.33 < 256x32x4 14.73 < 64x32x16 15.31 < 256x16x8 16.44 < 512x16x4 17.27)
+#define SPBLA_CT_T 128
+#define SPBLA_CT_I 32
+#define SPBLA_CT_B 8
+#endif
+constexpr int kCThreads = SPBLA_CT_T, kCItems = SPBLA_CT_I, kCMinB = SPBLA_CT_B;
+constexpr uint32_t kCT = kCThreads * kCItems;  // 4096 elements per tile
 constexpr uint32_t kCStage = 1024;             // rows of a tile staged in smem
 
 __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
@@ -1367,7 +1374,7 @@ __global__ void tile_deps_kernel(const uint64_t* __restrict__ src_lo, uint64_t n
     }
 }
 
-__global__ void __launch_bounds__(kCThreads, 4)
+__global__ void __launch_bounds__(kCThreads, kCMinB)
 compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint64_t* __restrict__ rowptr,
                        const uint32_t* __restrict__ tile_row, const uint2* __restrict__ wait_range,
                        idx_t nrows, uint64_t nnz, uint32_t* flags, uint32_t* ticket) {
@@ -1732,7 +1739,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
         tile_rows_kernel<<<gb, 256, 0, st>>>(rowptr.p, soff.p, nrows, ntiles, tile_row, src_lo.p);
         tile_deps_kernel<<<(unsigned)std::min<uint64_t>(ceil_div(ntiles, 256), uint64_t(nsm) * 8), 256, 0, st>>>(
             src_lo.p, ntiles, nnz, wait_range.p);
-        compact_inplace_kernel<<<nsm * 8, kCThreads, 0, st>>>(scratch.p, soff.p, rowptr.p, tile_row, wait_range.p,
+        compact_inplace_kernel<<<nsm * kCMinB * 2, kCThreads, 0, st>>>(scratch.p, soff.p, rowptr.p, tile_row, wait_range.p,
                                                              nrows, nnz, flags.p, flags.p + ntiles);
         count_launch(2);
         ktime_end(t);
