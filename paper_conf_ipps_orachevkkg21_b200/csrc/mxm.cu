@@ -77,40 +77,59 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
                 }
             }
         }
-        const uint32_t trips = __reduce_max_sync(0xffffffffu, valid ? uint32_t((e - b + kGroup - 1) / kGroup) : 0u);
+        // kR entries per lane per trip (entry b + 8*(kR*it + j) + g): all kR
+        // colidx loads, then all kR B-row records, are in flight together
+        constexpr int kR = 4;
+        const uint32_t trips =
+            __reduce_max_sync(0xffffffffu, valid ? uint32_t((e - b + kGroup * kR - 1) / (kGroup * kR)) : 0u);
         for (uint32_t it = 0; it < trips; ++it) {
-            const off_t64 p = b + it * kGroup + g;
-            uint32_t len = 0;
-            uint64_t ptr = 0;
-            if (valid && p < e) {
-                const idx_t k = A.colidx[p];
-                if (INFO) {
-                    const uint4 bi = binfo[k];  // span (0xFFFFFFFF, 0) when empty: neutral
-                    len = bi.y;
-                    ptr = reinterpret_cast<uint64_t>(bci + bi.x);
-                    lo = min(lo, bi.z);
-                    hi = max(hi, bi.w);
-                } else {
-                    const off_t64 x = brp[k], y = brp[k + 1];
-                    const uint2 sp = bspan[k];  // (0xFFFFFFFF, 0) when empty: neutral
-                    len = uint32_t(y - x);
-                    ptr = reinterpret_cast<uint64_t>(bci + x);
-                    lo = min(lo, sp.x);
-                    hi = max(hi, sp.y);
+            idx_t kk[kR];
+#pragma unroll
+            for (int j = 0; j < kR; ++j) {
+                const off_t64 p = b + (uint64_t(it) * kR + j) * kGroup + g;
+                kk[j] = (valid && p < e) ? A.colidx[p] : 0xFFFFFFFFu;
+            }
+            uint32_t len[kR];
+            uint64_t ptr[kR];
+#pragma unroll
+            for (int j = 0; j < kR; ++j) {
+                len[j] = 0;
+                ptr[j] = 0;
+                if (kk[j] != 0xFFFFFFFFu) {
+                    const idx_t k = kk[j];
+                    if (INFO) {
+                        const uint4 bi = binfo[k];  // span (0xFFFFFFFF, 0) when empty: neutral
+                        len[j] = bi.y;
+                        ptr[j] = reinterpret_cast<uint64_t>(bci + bi.x);
+                        lo = min(lo, bi.z);
+                        hi = max(hi, bi.w);
+                    } else {
+                        const off_t64 x = brp[k], y = brp[k + 1];
+                        const uint2 sp = bspan[k];  // (0xFFFFFFFF, 0) when empty: neutral
+                        len[j] = uint32_t(y - x);
+                        ptr[j] = reinterpret_cast<uint64_t>(bci + x);
+                        lo = min(lo, sp.x);
+                        hi = max(hi, sp.y);
+                    }
                 }
             }
-            s += len;
-            // compacted position and inclusive length prefix inside the group
-            const uint32_t m = (__ballot_sync(0xffffffffu, len > 0) >> gshift) & 0xFFu;
-            uint32_t inc = len;
 #pragma unroll
-            for (int d = 1; d < kGroup; d <<= 1) {
-                const uint32_t t = __shfl_up_sync(0xffffffffu, inc, d, kGroup);
-                if (g >= unsigned(d)) inc += t;
+            for (int j = 0; j < kR; ++j) {
+                s += len[j];
+                // compacted position and inclusive length prefix inside the group
+                const uint32_t m = (__ballot_sync(0xffffffffu, len[j] > 0) >> gshift) & 0xFFu;
+                uint32_t inc = len[j];
+#pragma unroll
+                for (int d = 1; d < kGroup; d <<= 1) {
+                    const uint32_t t = __shfl_up_sync(0xffffffffu, inc, d, kGroup);
+                    if (g >= unsigned(d)) inc += t;
+                }
+                if (len[j])
+                    drow[cn + __popc(m & ((1u << g) - 1u))] =
+                        make_uint4(uint32_t(ptr[j]), uint32_t(ptr[j] >> 32), len[j], cl + inc);
+                cn += __popc(m);
+                cl += __shfl_sync(0xffffffffu, inc, kGroup - 1, kGroup);
             }
-            if (len) drow[cn + __popc(m & ((1u << g) - 1u))] = make_uint4(uint32_t(ptr), uint32_t(ptr >> 32), len, cl + inc);
-            cn += __popc(m);
-            cl += __shfl_sync(0xffffffffu, inc, kGroup - 1, kGroup);
         }
         // row totals and column span (segments are sorted: first / last
         // entries), the span used by the hash and bitmap bins of the engine
