@@ -1519,6 +1519,8 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
     static_assert(PERSM * T <= 2048, #NAME " threads");
 // <threads, ub limit, overflow list, overflow buckets, descriptor batch, blocks/SM, loads per thread,
 //  dedup in pass B (else re-sort in pass A)>
+// (round-2 sweep on configs[4], tools/sweep_*.sh: 6 loads per thread for H1, H2, H6 -0.6 ms; 8 loads
+//  or 5 for H3-H5, 1024 threads for H5 all slower)
 // (expected per row at mean load 8 with 16 slots: list ~ub/1500, buckets ~ub/2000)
 #define HBIN(NAME, ...) HBIN_(NAME, __VA_ARGS__)
 #ifndef H0_CFG  // (overridable for tools/sweep.sh)
@@ -1526,11 +1528,11 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
 #endif
 HBIN(H0, H0_CFG)
 #ifndef H1_CFG  // (overridable for tools/sweep.sh)
-#define H1_CFG 32, kH1, 32, 16, 32, 24, 4, false
+#define H1_CFG 32, kH1, 32, 16, 32, 24, 6, false
 #endif
 HBIN(H1, H1_CFG)
 #ifndef H2_CFG  // (overridable for tools/sweep.sh)
-#define H2_CFG 64, kH2, 32, 16, 64, 16, 4, false
+#define H2_CFG 64, kH2, 32, 16, 64, 16, 6, false
 #endif
 HBIN(H2, H2_CFG)
 #ifndef H3_CFG  // (overridable for tools/sweep.sh)
@@ -1546,7 +1548,7 @@ HBIN(H4, H4_CFG)
 #endif
 HBIN(H5, H5_CFG)
 #ifndef H6_CFG  // (overridable for tools/sweep.sh)
-#define H6_CFG 1024, kH6, 192, 96, 384, 1, 4, true
+#define H6_CFG 1024, kH6, 192, 96, 384, 1, 6, true
 #endif
 HBIN(H6, H6_CFG)
 #define HASHK(N, KIND) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U, N##_DB, KIND>

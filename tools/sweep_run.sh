@@ -5,7 +5,7 @@ O=gpurun_out/sweep; mkdir -p $O; : > $O/summary.txt
 for so in paper_conf_ipps_orachevkkg21_b200/variants/libspbla_*.so; do
   name=$(basename $so .so); name=${name#libspbla_}
   for wl in ${WLS:-rmat22_ef32}; do
-    SPBLA_LIB_PATH=$PWD/$so timeout 300 python bench.py --workload $wl --no-cpu-baseline --no-e2e --steps 3 > $O/$name.$wl.json 2> $O/$name.$wl.err
+    SPBLA_LIB_PATH=$PWD/$so timeout 300 python bench.py --workload $wl --no-cpu-baseline --no-e2e --no-aux --steps 3 > $O/$name.$wl.json 2> $O/$name.$wl.err
     python -c "
 import json
 d=json.load(open('$O/$name.$wl.json'))
