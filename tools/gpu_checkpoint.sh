@@ -7,8 +7,8 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.used --format=csv > $
 timeout 1200 python -m pytest tests -m gpu -q > $O/pytest_gpu.txt 2>&1; tail -2 $O/pytest_gpu.txt
 timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; cut -c1-200 $O/bench.json
 timeout 600 python bench.py --impl reference > $O/bench_ref.json 2> $O/bench_ref.err; cut -c1-160 $O/bench_ref.json
-SPBLA_DIST_BACKEND=gloo timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 2 --warmup 3 --workload rmat20_ef16 --no-cpu-baseline > $O/bench_2rank_gloo.json 2> $O/bench_2rank_gloo.err; cut -c1-200 $O/bench_2rank_gloo.json
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_launch_bench.log 2>&1
+SPBLA_DIST_BACKEND=gloo timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 2 --warmup 3 --workload rmat20_ef16 --no-cpu-baseline --no-aux > $O/bench_2rank_gloo.json 2> $O/bench_2rank_gloo.err; cut -c1-200 $O/bench_2rank_gloo.json
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --no-aux > $O/ncu_launch_bench.log 2>&1
 # ncu --set full of the dominant kernels of one MxM of configs[4] (skip 1 = Build's launch)
 for kv in "compact:compact_inplace" "H4:hash_bin_kernel<.int.256,..unsigned.int.1024," "H5:hash_bin_kernel<.int.512,..unsigned.int.2560,"; do
   tag=${kv%%:*}; rx=${kv#*:}
