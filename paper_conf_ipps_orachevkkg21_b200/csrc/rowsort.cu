@@ -70,7 +70,11 @@ enum {
 };
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 // hash bins: ub limits (each sized so its tables fit the residency below)
-constexpr uint64_t kH0 = 512, kH1 = 1024, kH2 = 2048, kH3 = 4096, kH4 = 8192, kH5 = 20480, kH6 = 40960;
+#ifndef SPBLA_HB  // hash-bin ub limits (overridable for a sweep)
+#define SPBLA_HB 512, 1024, 2048, 4096, 8192, 20480, 40960
+#endif
+constexpr uint64_t kHB[7] = {SPBLA_HB};
+constexpr uint64_t kH0 = kHB[0], kH1 = kHB[1], kH2 = kHB[2], kH3 = kHB[3], kH4 = kHB[4], kH5 = kHB[5], kH6 = kHB[6];
 constexpr uint32_t kDenseBits = 3u << 19;      // bitmap window: 1.5 Mi columns, 192 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
