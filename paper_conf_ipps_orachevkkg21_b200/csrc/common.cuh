@@ -153,7 +153,7 @@ struct SegSource {
 // range (nullable): per-row [min col, max col] of the row's segments, needed
 // (and computed by MxM) for rows with ub > kRangeMinUb; null means [0, ncols).
 #ifndef SPBLA_WARP_MAX
-#define SPBLA_WARP_MAX 256
+#define SPBLA_WARP_MAX 128  // (rows of 129-256 products: the 32-thread hash bin H0; duplicate-heavy ones: W8)
 #endif
 constexpr uint64_t kRangeMinUb = SPBLA_WARP_MAX;
 // Bit 63 of a row's ub: the producer expects the row to be duplicate-heavy

@@ -1124,7 +1124,9 @@ __global__ void bin_count_kernel(const uint64_t* __restrict__ ub, const uint2* _
         // small bitmap windows skips the hash bins: its duplicates would
         // overflow the 16-slot buckets and send it to the same bitmap kernel
         // after a wasted gather
-        if ((uf & kUbDupFlag) && b >= BIN_H0 && b <= BIN_H6 && range && range[r].y - range[r].x < kSmallSpan)
+        if ((uf & kUbDupFlag) && u <= 256)  // (the warp bitonic bin is indifferent to duplicates)
+            b = u <= 32 ? BIN_W1 : u <= 64 ? BIN_W2 : u <= 128 ? BIN_W4 : BIN_W8;
+        else if ((uf & kUbDupFlag) && b >= BIN_H0 && b <= BIN_H6 && range && range[r].y - range[r].x < kSmallSpan)
             b = BIN_DUP;
         bin[r] = uint8_t(b);
         if (b == BIN_EMPTY) counts[r] = 0;
