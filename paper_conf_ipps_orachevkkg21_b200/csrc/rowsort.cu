@@ -1534,11 +1534,11 @@ constexpr size_t hash_smem(uint32_t threads, uint32_t batch, uint32_t buckets, u
 #endif
 HBIN(H0, H0_CFG)
 #ifndef H1_CFG  // (overridable for tools/sweep.sh)
-#define H1_CFG 32, kH1, 32, 16, 32, 24, 6, false
+#define H1_CFG 32, kH1, 32, 16, 32, 28, 6, false
 #endif
 HBIN(H1, H1_CFG)
 #ifndef H2_CFG  // (overridable for tools/sweep.sh)
-#define H2_CFG 64, kH2, 32, 16, 64, 16, 6, false
+#define H2_CFG 64, kH2, 32, 16, 64, 18, 6, false
 #endif
 HBIN(H2, H2_CFG)
 #ifndef H3_CFG  // (overridable for tools/sweep.sh)
