@@ -216,6 +216,16 @@ spbla_Status spbla_Matrix_Reduce(spbla_Matrix V, spbla_Matrix M, uint32_t hints)
  * receives the number of C += C x C evaluations, the last one included. */
 spbla_Status spbla_TransitiveClosure(spbla_Matrix C, int* iterations, uint32_t hints);
 
+/* Incremental transitive closure (§I l.117, l.126: an RPQ/CFPQ index
+ * is updated by adding edges to an already closed relation): C must be
+ * square and transitively closed (not checked), D the new edges (same
+ * shape, may alias nothing but may overlap C); C is replaced by the closure
+ * of C + D, computed semi-naively from the new entries (R11).
+ * *iterations (nullable) receives the number of closure steps evaluated,
+ * the confirming one included (0 when D adds no entry).  Errors: DIM_MISMATCH
+ * on shapes, INVALID_ARGUMENT on a non-owning C. */
+spbla_Status spbla_TransitiveClosureIncremental(spbla_Matrix C, spbla_Matrix D, int* iterations, uint32_t hints);
+
 #ifdef __cplusplus
 }
 #endif

@@ -23,7 +23,7 @@ __all__ = [
     "SpblaError", "Initialize", "Finalize", "SetStream", "Synchronize", "memory_stats",
     "reset_peak_memory", "launch_count", "reset_launch_count", "Matrix", "Matrix_New",
     "Matrix_Build", "Matrix_ExtractPairs", "MxM", "Matrix_EWiseAdd", "Kronecker",
-    "Matrix_Transpose", "Matrix_ExtractSubMatrix", "Matrix_Reduce", "TransitiveClosure",
+    "Matrix_Transpose", "Matrix_ExtractSubMatrix", "Matrix_Reduce", "TransitiveClosure", "TransitiveClosureIncremental",
 ]
 
 
@@ -387,6 +387,14 @@ def Matrix_Reduce(V: Matrix, M: Matrix):
 def TransitiveClosure(C: Matrix) -> int:
     it = ctypes.c_int(0)
     _check(_lib().spbla_TransitiveClosure(C.handle, ctypes.byref(it), 0), "spbla_TransitiveClosure")
+    return int(it.value)
+
+
+def TransitiveClosureIncremental(C: Matrix, D: Matrix) -> int:
+    """C (transitively closed) <- closure(C + D); returns the closure steps."""
+    it = ctypes.c_int(0)
+    _check(_lib().spbla_TransitiveClosureIncremental(C.handle, D.handle, ctypes.byref(it), 0),
+           "spbla_TransitiveClosureIncremental")
     return int(it.value)
 
 

@@ -53,6 +53,7 @@ SIGNATURES = {
     "spbla_Matrix_ExtractSubMatrix": (_int, [_vp, _vp, _u32, _u32, _u32, _u32, _u32]),
     "spbla_Matrix_Reduce": (_int, [_vp, _vp, _u32]),
     "spbla_TransitiveClosure": (_int, [_vp, ctypes.POINTER(_int), _u32]),
+    "spbla_TransitiveClosureIncremental": (_int, [_vp, _vp, ctypes.POINTER(_int), _u32]),
 }
 
 HINT_NO = 0

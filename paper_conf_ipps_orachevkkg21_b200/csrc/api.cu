@@ -9,6 +9,7 @@
 namespace spbla {
 void mxm(Matrix* C, const Matrix* A, const Matrix* B, bool accumulate, uint32_t dup_ratio = 0);
 int transitive_closure(Matrix* C);
+int transitive_closure_incremental(Matrix* C, const Matrix* D);
 void ewise_add(Matrix* C, const Matrix* A, const Matrix* B);
 void kronecker(Matrix* K, const Matrix* A, const Matrix* B);
 void transpose(Matrix* T, const Matrix* M);
@@ -397,6 +398,17 @@ spbla_Status spbla_TransitiveClosure(spbla_Matrix C, int* iterations, uint32_t h
         NEED(C, "null matrix");
         NEED(C->owned, "closure: matrix is a non-owning view");
         int it = transitive_closure(C);
+        if (iterations) *iterations = it;
+    });
+}
+
+spbla_Status spbla_TransitiveClosureIncremental(spbla_Matrix C, spbla_Matrix D, int* iterations, uint32_t hints) {
+    (void)hints;
+    return guarded([&] {
+        require_init();
+        NEED(C && D, "null matrix");
+        NEED(C->owned, "closure: matrix is a non-owning view");
+        int it = transitive_closure_incremental(C, D);
         if (iterations) *iterations = it;
     });
 }

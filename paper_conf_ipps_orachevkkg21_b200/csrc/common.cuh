@@ -159,6 +159,10 @@ constexpr uint64_t kRangeMinUb = SPBLA_WARP_MAX;
 // Bit 63 of a row's ub: the producer expects the row to be duplicate-heavy
 // (closure steps: products >> the row's current length); the engine masks it.
 constexpr uint64_t kUbDupFlag = uint64_t(1) << 63;
+// Bit 62: the row's only segment is already a sorted duplicate-free row (the
+// accumulate input C[r] of a row with no B products): the engine copies it.
+constexpr uint64_t kUbCopyFlag = uint64_t(1) << 62;
+constexpr uint64_t kUbValue = kUbCopyFlag - 1;  // the count without the flags
 void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, const uint2* range,
                 Matrix* out);
 

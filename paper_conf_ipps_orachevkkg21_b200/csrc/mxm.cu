@@ -143,7 +143,9 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
             // dup_ratio (closure steps): products far above the row's current
             // length mean mostly repeated columns (C[k] largely inside C[r])
             const bool dup = dup_ratio && s > kRangeMinUb && s > uint64_t(dup_ratio) * lcr;
-            ub[r] = s | (dup ? kUbDupFlag : 0);
+            // (a row whose only products are its accumulate input: a copy)
+            const bool copy = crp && cn == 1 && s == lcr;
+            ub[r] = s | (dup ? kUbDupFlag : 0) | (copy ? kUbCopyFlag : 0);
             nseg[r] = cn;
             if (s > kRangeMinUb) range[r] = make_uint2(lo, hi);
         }
@@ -258,15 +260,12 @@ void swap_storage(Matrix* a, Matrix* b) { std::swap(*a, *b); }
 // iterates and the iteration count are those of the plain loop.
 constexpr uint64_t kSemiNaiveDiv = 8;
 
-int transitive_closure(Matrix* C) {
-    if (C->nrows != C->ncols) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "closure: matrix must be square");
+// The loop after the first step: prev = C_{k-1}, C = C_k, with
+// C_{k-1} C_{k-1} inside C_k; plain squaring or the semi-naive step
+// (R11) by the share of new entries; returns the steps evaluated.
+static int closure_steps(Matrix* C, OwnedMatrix& prev) {
     const idx_t n = C->nrows;
-    OwnedMatrix prev(n, n);  // C_{k-1}
-    matrix_duplicate(C, &prev.m);
-    // closure steps: rows whose products exceed kClosureDupRatio x their
-    // current length are routed to the bitmap kernel (DESIGN.md §4.2)
-    mxm(C, C, C, true, kClosureDupRatio);
-    int it = 1;
+    int it = 0;
     while (C->nnz != prev.m.nnz) {  // C only grows: equal nnz <=> fixed point
         const uint64_t added = C->nnz - prev.m.nnz;
         if (added * kSemiNaiveDiv < C->nnz) {
@@ -287,6 +286,37 @@ int transitive_closure(Matrix* C) {
         ++it;
     }
     return it;
+}
+
+int transitive_closure(Matrix* C) {
+    if (C->nrows != C->ncols) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "closure: matrix must be square");
+    const idx_t n = C->nrows;
+    OwnedMatrix prev(n, n);  // C_{k-1}
+    matrix_duplicate(C, &prev.m);
+    // closure steps: rows whose products exceed kClosureDupRatio x their
+    // current length are routed to the bitmap kernel (DESIGN.md §4.2)
+    mxm(C, C, C, true, kClosureDupRatio);
+    return 1 + closure_steps(C, prev);
+}
+
+// Incremental closure (§I l.117, l.126: CFPQ/RPQ index updates add
+// edges to an already closed relation): C is transitively closed, D holds
+// new edges; C becomes the closure of C + D.  With C_{-1} = C (closed: C C is
+// inside C) and C_0 = C + D, the loop above applies from the start; its first
+// step is semi-naive with Delta_0 = D \ C (the new entries only).  Returns the
+// closure steps evaluated, the confirming one included (0 when D adds
+// nothing).
+void ewise_add(Matrix* C, const Matrix* A, const Matrix* B);
+
+int transitive_closure_incremental(Matrix* C, const Matrix* D) {
+    if (C->nrows != C->ncols) SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "closure: matrix must be square");
+    if (D->nrows != C->nrows || D->ncols != C->ncols)
+        SPBLA_THROW(SPBLA_STATUS_DIM_MISMATCH, "incremental closure: D must have C's shape");
+    const idx_t n = C->nrows;
+    OwnedMatrix prev(n, n);
+    matrix_duplicate(C, &prev.m);
+    ewise_add(C, C, D);  // C_0 = C + D
+    return closure_steps(C, prev);
 }
 
 }  // namespace spbla

@@ -62,11 +62,12 @@ __shared__ unsigned long long s_probe_ext[12];
 #define PROBE(i) do {} while (0)
 #define PROBE_PRINT(tag, u, ns) do {} while (0)
 #endif
-constexpr int kNumBins = 14;
+constexpr int kNumBins = 15;
 enum {
     BIN_EMPTY = 0, BIN_W1 = 1, BIN_W2, BIN_W4, BIN_W8, BIN_H0,
     BIN_H1 = 6, BIN_H2, BIN_H3, BIN_H4, BIN_H5, BIN_H6, BIN_DENSE = 12,
-    BIN_DUP = 13  // rows flagged duplicate-heavy (kUbDupFlag): straight to the small bitmap kernel
+    BIN_DUP = 13,  // rows flagged duplicate-heavy (kUbDupFlag): straight to the small bitmap kernel
+    BIN_COPY = 14  // rows flagged copy-only (kUbCopyFlag): their single segment is the output
 };
 constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 // hash bins: ub limits (each sized so its tables fit the residency below)
@@ -994,7 +995,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         // window-w emission writes below the start of slice w+1 (distinct <=
         // products), so it never overwrites an unread slice.  Two gathers
         // and a slice pass per row, whatever the number of windows.
-        const uint64_t prods = ub[r] & ~kUbDupFlag;
+        const uint64_t prods = ub[r] & kUbValue;
         const bool part = nwin > 3 && prods <= soff[r + 1] - soff[r] && nwin < 2 * BATCH;
         uint32_t* wcur = bm;               // (partition mode, during the gathers) per-window cursors
         uint32_t* wbeg = bm + kWords / 2;  // ... and slice starts (nwin + 1 entries)
@@ -1117,19 +1118,22 @@ __global__ void bin_count_kernel(const uint64_t* __restrict__ ub, const uint2* _
     __syncthreads();
     for (size_t r = blockIdx.x * size_t(blockDim.x) + threadIdx.x; r < nrows;
          r += size_t(gridDim.x) * blockDim.x) {
-        const uint64_t uf = ub[r], u = uf & ~kUbDupFlag;
+        const uint64_t uf = ub[r], u = uf & kUbValue;
         cap[r] = u < ncols ? u : uint64_t(ncols);
         int b = bin_of(u);
         // a duplicate-heavy row (flagged by the producer) whose span fits two
         // small bitmap windows skips the hash bins: its duplicates would
         // overflow the 16-slot buckets and send it to the same bitmap kernel
         // after a wasted gather
-        if ((uf & kUbDupFlag) && u <= 256)  // (the warp bitonic bin is indifferent to duplicates)
+        if (uf & kUbCopyFlag)  // (exact count: the copy kernel writes the row as it is)
+            b = BIN_COPY;
+        else if ((uf & kUbDupFlag) && u <= 256)  // (the warp bitonic bin is indifferent to duplicates)
             b = u <= 32 ? BIN_W1 : u <= 64 ? BIN_W2 : u <= 128 ? BIN_W4 : BIN_W8;
         else if ((uf & kUbDupFlag) && b >= BIN_H0 && b <= BIN_H6 && range && range[r].y - range[r].x < kSmallSpan)
             b = BIN_DUP;
         bin[r] = uint8_t(b);
         if (b == BIN_EMPTY) counts[r] = 0;
+        if (b == BIN_COPY) counts[r] = uint32_t(u);
         atomicAdd(&sh[b], 1u);
     }
     __syncthreads();
@@ -1181,7 +1185,7 @@ __global__ void make_recs_kernel(SegSource src, const idx_t* __restrict__ rows, 
         const idx_t r = rows[i];
         RowRec x;
         x.r = r;
-        x.u = uint32_t(min(ub[r] & ~kUbDupFlag, uint64_t(0xFFFFFFFFu)));
+        x.u = uint32_t(min(ub[r] & kUbValue, uint64_t(0xFFFFFFFFu)));
         if (range) {
             const uint2 rg = range[r];
             x.clo = rg.x;
@@ -1281,6 +1285,23 @@ warp_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* _
         for (int e = 0; e < E; ++e)
             if (uniq[e]) out[o++] = x[e];
         if (lane == 31) counts[r] = inc;
+    }
+}
+
+// ---- 4d. copy bin: rows whose only segment is the output (accumulate input
+// of a row without products, e.g. most rows of C += C Delta): warp per row
+__global__ void __launch_bounds__(256)
+copy_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ binoff,
+                idx_t* __restrict__ scratch, const uint64_t* __restrict__ soff) {
+    const unsigned lane = lane_id();
+    const uint32_t lo = binoff[BIN_COPY], hi = binoff[BIN_COPY + 1];
+    const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+    for (uint32_t t = lo + blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); t < hi; t += nwarps) {
+        const idx_t r = rows[t];
+        uint32_t len;
+        const idx_t* p = get_seg(src, r, 0, len);
+        idx_t* o = scratch + soff[r];
+        for (uint32_t i = lane; i < len; i += 32) o[i] = p[i];
     }
 }
 
@@ -1612,15 +1633,15 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     DevBuf<uint64_t> soff(size_t(nrows) + 1);
     DevBuf<uint8_t> bin(nrows);
     DevBuf<uint32_t> counts(nrows);
-    // meta: hist[14] binoff[15] cursor[14] work[9] ovf[4] work2[1] work3[1]
+    // meta: hist[15] binoff[16] cursor[15] work[9] ovf[4] work2[1] work3[1]
     DevBuf<uint32_t> meta(64);
     uint32_t* hist = meta.p;
-    uint32_t* binoff = meta.p + 14;
-    uint32_t* cursor = meta.p + 29;
-    uint32_t* work = meta.p + 43;
-    uint32_t* ovf = meta.p + 52;  // fallback lists: [0, ovf[1]) and [nrows, ovf[3])
-    uint32_t* work2 = meta.p + 56;
-    uint32_t* work3 = meta.p + 57;
+    uint32_t* binoff = meta.p + 15;
+    uint32_t* cursor = meta.p + 31;
+    uint32_t* work = meta.p + 46;
+    uint32_t* ovf = meta.p + 55;  // fallback lists: [0, ovf[1]) and [nrows, ovf[3])
+    uint32_t* work2 = meta.p + 59;
+    uint32_t* work3 = meta.p + 60;
     memset_async(meta.p, 0, meta.n * sizeof(uint32_t));
     {
         const uint32_t lst1[2] = {nrows, nrows};
@@ -1669,6 +1690,14 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
         count_launch();
     }
     ktime_end(t);
+    if (hcnt[BIN_COPY]) {
+        t = ktime_begin("warp_bins", st);
+        copy_bin_kernel<<<std::min<uint32_t>(nsm * 8, (hcnt[BIN_COPY] + 7) / 8), 256, 0, st>>>(src, rows.p, binoff,
+                                                                                           scratch.p, soff.p);
+        count_launch();
+        ktime_end(t);
+        check_launch("copy_bin_kernel");
+    }
     t = ktime_begin("dense_ovf", st);
     if (hcnt[BIN_DUP]) {  // duplicate-heavy rows flagged by the producer
         SDENSE<<<std::min<uint32_t>(nsm * kSDPerSM, hcnt[BIN_DUP]), 256, kSDSmem, st>>>(

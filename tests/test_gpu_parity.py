@@ -370,3 +370,31 @@ def test_mxm_heavy_rows_wide_span_partition(sp):
     A, OA = both_from_pairs(sp, 40, k, ra, ca)
     B, OB = both_from_pairs(sp, k, ncols, rb, cb)
     assert_same(sp.mxm(A, B), oracle.mxm(OA, OB), "heavy rows over 2^26 columns")
+
+
+@pytest.mark.parametrize("n,p,extra,seed", [(1 << 11, 0.25, 300, 90), (1 << 13, 0.1, 2000, 91), (700, 0.5, 0, 92)])
+def test_incremental_closure(sp, n, p, extra, seed):
+    """spbla_TransitiveClosureIncremental: C = closure(G), then new edges D
+    (some inside C already); C becomes closure(G + D) -- the oracle's closure
+    of the union -- and D inside C leaves C unchanged with 0 steps."""
+    (r0, c0), (r1, c1) = spgen.labeled_dag(n, p, seed=seed)
+    rg = np.concatenate([r0.numpy(), r1.numpy()])
+    cg = np.concatenate([c0.numpy(), c1.numpy()])
+    G, OG = both_from_pairs(sp, n, n, rg, cg)
+    C, _ = sp.closure(G)
+    OC, _ = oracle.closure(OG)
+    assert_same(C, OC, "closure(G)")
+    rng = np.random.default_rng(seed)
+    rd = rng.integers(1, n, extra).astype(np.uint32)
+    cd = (rng.integers(0, 1 << 30, extra) % np.maximum(rd, 1)).astype(np.uint32)  # DAG edges v -> u < v
+    rd = np.concatenate([rd, rg[:50]]).astype(np.uint32)  # plus edges C already has
+    cd = np.concatenate([cd, cg[:50]]).astype(np.uint32)
+    D, OD = both_from_pairs(sp, n, n, rd, cd)
+    it = sp.TransitiveClosureIncremental(C, D)
+    want, _ = oracle.closure(oracle.ewise_add(OG, OD))
+    assert_same(C, want, "closure(G + D) incrementally")
+    assert (it == 0) == (extra == 0)
+    # D inside C: nothing changes
+    E, _ = both_from_pairs(sp, n, n, rg[:100], cg[:100])
+    assert sp.TransitiveClosureIncremental(C, E) == 0
+    assert_same(C, want, "unchanged by edges already present")
