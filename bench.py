@@ -486,6 +486,7 @@ def main():
               ("mxm_ub", "warp_bins", "H0", "H1", "H2", "H3", "H4", "H5", "H6", "dense", "dense_ovf", "compact")}
     sp.set_kernel_timing(False)
     peak_mem = sp.memory_stats()[1]
+    pool_reserved = sp.pool_stats()[0]  # (device memory the pools hold, incl. the size-class cache)
     red_dev = "cpu" if world > 1 and dist.get_backend() == "gloo" else "cuda"
     tot = torch.tensor([sum(step_ms), peak_mem, nnzC_local, launches], dtype=torch.float64, device=red_dev)
     if world > 1:
@@ -619,6 +620,7 @@ def main():
                        "l2": "A larger than L2 (126 MB) and a 256 MB write between timed steps",
                        "peak_mem_gb": peak_mem_max / 1e9},
             "peak_mem_gb": peak_mem_max / 1e9,
+            "pool_reserved_gb_rank0": pool_reserved / 1e9,
             "gpu_launches": launches_all,
             "clocks": clk,
             "roofline": roof,
