@@ -30,20 +30,40 @@ namespace spbla {
 namespace {
 
 #ifndef SPBLA_EW_THREADS  // (overridable for a sweep)
-#define SPBLA_EW_THREADS 512
+#define SPBLA_EW_THREADS 256
+#endif
+#ifndef SPBLA_EW_ITEMS
+#define SPBLA_EW_ITEMS 16
 #endif
 constexpr int kThreads = SPBLA_EW_THREADS;
-constexpr int kMinBlocks = 1536 / kThreads;  // 1536 threads per SM at ~30 KB smem per 2048 items
-constexpr int kItems = 8;
-constexpr uint32_t kTile = kThreads * kItems;  // merged items per tile (4096 at 512 threads)
-// padded smem indices: threads own kItems consecutive positions, so a plain
-// layout puts the lanes of a warp kItems words apart (8- to 16-way bank
-// conflicts); one pad word per 16 (keys, 64-bit) / 32 (marks, output) words
-// spreads them over all banks
-__device__ __forceinline__ uint32_t KI(uint32_t p) { return p + (p >> 4); }
+constexpr int kItems = SPBLA_EW_ITEMS;  // merged items per thread (<= 32: one dup-mask word)
+constexpr uint32_t kTile = kThreads * kItems;  // merged items per tile (4096)
+#ifndef SPBLA_EW_ROWS
+#define SPBLA_EW_ROWS 1024
+#endif
+constexpr uint32_t kRowStage = SPBLA_EW_ROWS;  // rows of a tile staged in smem (else read from global)
+static_assert(kItems <= 32, "dup mask");
+// padded smem index: threads own kItems consecutive positions, so a plain
+// layout puts the lanes of a warp kItems words apart; one pad word per 32
+// spreads them over the banks
 __device__ __forceinline__ uint32_t OI(uint32_t p) { return p + (p >> 5); }
-constexpr uint32_t kKeyWords = kTile + kTile / 16, kOutWords = kTile + kTile / 32 + 1;
-constexpr size_t kMergeSmem = size_t(kKeyWords) * 8 + size_t(kOutWords) * 4 + (kTile + 1) * 2;
+constexpr uint32_t kColWords = kTile + kTile / 32 + 1;
+constexpr size_t kMergeSmem = size_t(kTile + 4 + kColWords) * 4 + size_t(2 * (kRowStage + 1)) * 2;
+static_assert(kTile <= 65535, "16-bit local row offsets");
+static_assert(2 * kThreads <= kTile, "duplicate scan words alias the staged columns");
+#ifndef SPBLA_EW_LB
+#define SPBLA_EW_LB 1
+#endif
+#ifndef SPBLA_EW_UNROLL
+#define SPBLA_EW_UNROLL 1
+#endif
+constexpr int kLB = SPBLA_EW_LB;  // look-back statuses per lane per round trip
+constexpr int kUnroll = SPBLA_EW_UNROLL;  // merge-loop copies
+constexpr int kChunks = (kTile / 4 + 4 + kThreads - 1) / kThreads;  // 16-B staging chunks per thread
+#ifndef SPBLA_EW_MINB
+#define SPBLA_EW_MINB (1536 / SPBLA_EW_THREADS)  // 40 registers at 256 threads (8 blocks spill)
+#endif
+constexpr int kMinBlocks = SPBLA_EW_MINB;
 constexpr uint64_t kFlagAgg = 1ull << 62;
 constexpr uint64_t kFlagPre = 2ull << 62;
 constexpr uint64_t kValMask = (1ull << 62) - 1;
@@ -105,21 +125,106 @@ __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
     return v;
 }
 
+// local offset of a row boundary v (global A or B position) in the tile's
+// range [x0, x0 + n)
+__device__ __forceinline__ uint32_t tile_seg(uint64_t v, uint64_t x0, uint32_t n) {
+    return v <= x0 ? 0u : uint32_t(min(v - x0, uint64_t(n)));
+}
+
+// Step 2 of the merge kernel: the calling thread's kItems merged positions
+// [k0, k1) into s_m; returns the duplicate mask (bit k: position k0 + k is a
+// B item equal to the A item before it).  STAGED: the tile rows' local
+// segment starts are in s_ra / s_rb, else they are read from global.
+template <bool STAGED>
+__device__ __forceinline__ uint32_t merge_thread(const MergeIn& m, const uint32_t* s_col, uint32_t* s_m,
+                                                 const uint16_t* s_ra, const uint16_t* s_rb, uint32_t r0,
+                                                 uint32_t nr, uint32_t na, uint32_t nb, uint32_t len,
+                                                 uint64_t a0, uint64_t b0, uint64_t prev) {
+    const uint32_t k0 = min(uint32_t(threadIdx.x) * kItems, len), k1 = min(k0 + kItems, len);
+    if (k0 >= k1) return 0u;
+    auto SA = [&](uint32_t i) -> uint32_t { return STAGED ? uint32_t(s_ra[i]) : tile_seg(m.rpa[r0 + i], a0, na); };
+    auto SB = [&](uint32_t i) -> uint32_t { return STAGED ? uint32_t(s_rb[i]) : tile_seg(m.rpb[r0 + i], b0, nb); };
+    // last tile row i in [lo, nr - 1] whose local merged start is <= p
+    auto find_row = [&](uint32_t lo, uint32_t p) -> uint32_t {
+        uint32_t hi = nr - 1;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi + 1) >> 1;
+            if (SA(mid) + SB(mid) <= p) lo = mid; else hi = mid - 1;
+        }
+        return lo;
+    };
+    uint32_t i = find_row(0, k0);
+    const uint32_t as = SA(i), bs = SB(i);
+    uint32_t aend = SA(i + 1), bend = SB(i + 1);
+    // merge-path split of local position k0 inside row i
+    uint32_t lo = max(as, k0 > bend ? k0 - bend : 0u), hi = min(aend, k0 - bs);
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_col[mid] <= s_col[na + k0 - 1 - mid]) lo = mid + 1; else hi = mid;
+    }
+    uint32_t ai = lo, bi = k0 - lo;
+    uint32_t nxt = aend + bend;
+    // A duplicate B item directly follows its equal A item in the merge
+    // (ties take A; rows are sorted and duplicate-free), so it is exactly an
+    // item equal to the previous merged item of its row.  `last`: that item
+    // (the row's last A item before k0 suffices: a B item before k0 is
+    // smaller than every later B item); ~0 is no column (ncols < 2^32).
+    uint32_t last = ai > as ? s_col[ai - 1] : (i == 0 ? uint32_t(prev) : ~0u);
+    uint32_t va = s_col[ai], vb = s_col[na + bi];
+    uint32_t dmask = 0;
+#pragma unroll kUnroll
+    for (uint32_t k = 0; k < k1 - k0; ++k) {
+        const uint32_t pos = k0 + k;
+        if (__builtin_expect(pos == nxt, 0)) {  // next non-empty row
+            ++i;
+            if (SA(i + 1) + SB(i + 1) <= pos) i = find_row(i + 1, pos);
+            aend = SA(i + 1);
+            bend = SB(i + 1);
+            nxt = aend + bend;
+            last = ~0u;
+        }
+        const bool takeA = ai < aend && (bi == bend || va <= vb);
+        const uint32_t c = takeA ? va : vb;
+        dmask |= uint32_t(c == last) << k;
+        last = c;
+        ai += takeA;
+        bi += !takeA;
+        const uint32_t nv = s_col[takeA ? ai : na + bi];
+        va = takeA ? nv : va;
+        vb = takeA ? vb : nv;
+        s_m[OI(pos)] = c;
+    }
+    return dmask;
+}
+
+// One tile of kTile merged items per block (ticket order).  The tile's A
+// range [a0, a1) and B range [b0, b1) (from the split kernel) are staged as
+// columns; every thread then merges kItems consecutive merged positions
+// sequentially, row by row: rows are the tile's per-row segments of A and B
+// (local offsets staged in smem), the thread's first row and its merge-path
+// split inside that row come from two binary searches, and a row change
+// only moves the segment ends (the local merged start of row i is the sum
+// of its A and B starts).  A B item is a duplicate iff it equals the last A
+// item taken in its row (ties take A first; for the tile's first row the A
+// item before the tile is tile_prev).  The merged columns go to smem at
+// their merged positions; a tile with duplicates (block-uniform test) then
+// closes the gaps in smem.  Kept counts: warp scans + one smem round; the
+// tile's output base: decoupled look-back by warp 0; 16-B coalesced stores.
 __global__ void __launch_bounds__(kThreads, kMinBlocks)
 ewise_merge_kernel(MergeIn m, uint64_t ntiles, const uint32_t* __restrict__ tile_row,
                    const uint64_t* __restrict__ tile_a, const uint32_t* __restrict__ tile_rlo,
                    const uint64_t* __restrict__ tile_prev, uint64_t* status, uint32_t* ticket,
                    idx_t* __restrict__ out, off_t64* __restrict__ rowptr) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    uint64_t* s_key = reinterpret_cast<uint64_t*>(smem_raw);    // [kTile] A keys [0, na), B keys [na, len)
-    uint32_t* s_out = reinterpret_cast<uint32_t*>(s_key + kKeyWords);  // kept columns in output order (OI)
-    uint16_t* s_dpre = reinterpret_cast<uint16_t*>(s_out + kOutWords);  // [kTile+1] duplicates before each position
-    __shared__ uint64_t sh[33];
+    uint32_t* s_col = reinterpret_cast<uint32_t*>(smem_raw);  // A cols [0, na), B cols [na, len) (+1 pad)
+    uint32_t* s_m = s_col + (kTile + 4);                         // merged columns at [OI(pos)]
+    uint16_t* s_ra = reinterpret_cast<uint16_t*>(s_m + kColWords);  // local A start of tile row i
+    uint16_t* s_rb = s_ra + (kRowStage + 1);                         // local B start of tile row i
+    uint32_t* s_tdup = s_col;            // (after the merge) duplicates before each thread
+    uint32_t* s_dmask = s_col + kThreads;  // (after the merge) each thread's duplicate mask
+    __shared__ uint32_t s_wdup[kThreads / 32];
     __shared__ uint32_t s_t;
     __shared__ uint64_t s_base;
-    uint32_t* s_mark = s_out;  // row marks (scratch until the output is staged)
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) s_mark[OI(threadIdx.x * kItems + k)] = 0u;
     if (threadIdx.x == 0) s_t = atomicAdd(ticket, 1u);  // ticket order: the look-back never waits on a later block
     __syncthreads();
     const uint64_t t = s_t;
@@ -129,144 +234,167 @@ ewise_merge_kernel(MergeIn m, uint64_t ntiles, const uint32_t* __restrict__ tile
     const uint64_t b0 = d0 - a0, b1 = d1 - a1;
     const uint32_t na = uint32_t(a1 - a0), nb = uint32_t(b1 - b0);
     const uint32_t r0 = tile_row[t], r1 = min(tile_row[t + 1], m.nrows - 1);
-    const uint64_t prevA = tile_prev[t];
-    // 1. stage the columns (coalesced) and, in the same round trip, mark the
-    //    first tile position of every row segment (0 = no mark; B marks are
-    //    offset by nrows + 1 so that no A row carries into the B part); a
-    //    max-scan then gives every position its row, ORed into the key
+    const uint32_t nr = r1 - r0 + 1;  // tile rows r0..r1; row nr's start is the tile end
+    const uint64_t prev = tile_prev[t];
+    uint32_t dmask;
+    // 1. stage the columns as aligned 16-B chunks (A's chunks, then B's;
+    //    all loads in flight before the first smem store) and the rows'
+    //    local segment starts, clamped to the tile
     {
-        idx_t cv[kItems];  // all loads in flight before the first smem store
+        const uintptr_t pa = reinterpret_cast<uintptr_t>(m.ca + a0), pb = reinterpret_cast<uintptr_t>(m.cb + b0);
+        const uint4* ga = reinterpret_cast<const uint4*>(pa & ~uintptr_t(15));
+        const uint4* gb = reinterpret_cast<const uint4*>(pb & ~uintptr_t(15));
+        const uint32_t offa = uint32_t(pa & 15) >> 2, offb = uint32_t(pb & 15) >> 2;
+        const uint32_t nca = na ? (offa + na + 3) >> 2 : 0u, ncb = nb ? (offb + nb + 3) >> 2 : 0u;
+        uint4 cv[kChunks];
 #pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            const uint32_t pos = k * kThreads + threadIdx.x;
-            cv[k] = pos < na ? m.ca[a0 + pos] : (pos < len ? m.cb[b0 + (pos - na)] : 0u);
+        for (int j = 0; j < kChunks; ++j) {
+            const uint32_t c = j * kThreads + threadIdx.x;
+            cv[j] = c < nca ? ga[c] : (c < nca + ncb ? gb[c - nca] : make_uint4(0, 0, 0, 0));
         }
 #pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            const uint32_t pos = k * kThreads + threadIdx.x;
-            if (pos < len) s_key[KI(pos)] = cv[k];
+        for (int j = 0; j < kChunks; ++j) {
+            const uint32_t c = j * kThreads + threadIdx.x;
+            if (c < nca + ncb) {
+                const bool isa = c < nca;
+                // smem position of the chunk's first word and the valid range
+                const int32_t e = isa ? int32_t(4 * c) - int32_t(offa) : int32_t(na + 4 * (c - nca)) - int32_t(offb);
+                const int32_t lo = isa ? 0 : int32_t(na), hi = isa ? int32_t(na) : int32_t(len);
+                const uint32_t w[4] = {cv[j].x, cv[j].y, cv[j].z, cv[j].w};
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (e + q >= lo && e + q < hi) s_col[e + q] = w[q];
+            }
         }
     }
-    const uint32_t boff = m.nrows + 1;
-#pragma unroll 1
-    for (uint32_t r = r0 + threadIdx.x; r <= r1; r += kThreads) {
-        const uint64_t ra = max(m.rpa[r], a0), rae = min(m.rpa[r + 1], a1);
-        const uint64_t rb = max(m.rpb[r], b0), rbe = min(m.rpb[r + 1], b1);
-        if (ra < rae) s_mark[OI(uint32_t(ra - a0))] = r + 1;
-        if (rb < rbe) s_mark[OI(na + uint32_t(rb - b0))] = boff + r + 1;
-    }
-    __syncthreads();
-    {
-        uint32_t v[kItems], run = 0;
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            run = max(run, s_mark[OI(threadIdx.x * kItems + k)]);
-            v[k] = run;
+    if (nr <= kRowStage) {
+        for (uint32_t i = threadIdx.x; i <= nr; i += kThreads) {
+            s_ra[i] = uint16_t(tile_seg(m.rpa[r0 + i], a0, na));
+            s_rb[i] = uint16_t(tile_seg(m.rpb[r0 + i], b0, nb));
         }
-        // block exclusive max-scan of the thread maxima
-        uint32_t inc = run;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, d);
-            if (int(lane_id()) >= d) inc = max(inc, y);
-        }
-        __shared__ uint32_t s_wmax[kThreads / 32];
-        if (lane_id() == 31) s_wmax[threadIdx.x >> 5] = inc;
         __syncthreads();
-        uint32_t carry = 0;
-        for (unsigned w = 0; w < (threadIdx.x >> 5); ++w) carry = max(carry, s_wmax[w]);
-        const uint32_t ex = max(carry, __shfl_up_sync(0xffffffffu, inc, 1) * (lane_id() > 0));
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            const uint32_t pos = threadIdx.x * kItems + k;
-            if (pos < len) {
-                uint32_t rr = max(ex, v[k]) - 1;
-                if (pos >= na) rr -= boff;
-                s_key[KI(pos)] |= uint64_t(rr) << 32;
-            }
-        }
+        dmask = merge_thread<true>(m, s_col, s_m, s_ra, s_rb, r0, nr, na, nb, len, a0, b0, prev);
+    } else {  // (many empty or single-item rows: row starts read from global)
+        __syncthreads();
+        dmask = merge_thread<false>(m, s_col, s_m, s_ra, s_rb, r0, nr, na, nb, len, a0, b0, prev);
     }
-    __syncthreads();
-    // 2. merge path per thread over the smem keys, kItems items each
     const uint32_t k0 = min(uint32_t(threadIdx.x) * kItems, len), k1 = min(k0 + kItems, len);
-    uint32_t lo = k0 > nb ? k0 - nb : 0, hi = min(k0, na);
-    while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (s_key[KI(mid)] <= s_key[KI(na + k0 - 1 - mid)]) lo = mid + 1; else hi = mid;
-    }
-    uint32_t ai = lo, bi = k0 - lo;
-    idx_t col[kItems];
-    uint32_t dmask = 0, ndup = 0;
+    // 3. duplicates before this thread (warp scan + one smem round); the
+    //    tile's kept count
+    const uint32_t ndup = __popc(dmask);
+    uint32_t inc = ndup;
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-        col[k] = 0;
-        if (k0 + k < k1) {
-            const bool takeA = ai < na && (bi == nb || s_key[KI(ai)] <= s_key[KI(na + bi)]);
-            if (takeA) {
-                col[k] = idx_t(s_key[KI(ai++)]);
-            } else {
-                const uint64_t kb = s_key[KI(na + bi++)];
-                const uint64_t pa = ai > 0 ? s_key[KI(ai - 1)] : prevA;
-                col[k] = idx_t(kb);
-                if (pa == kb) {
-                    dmask |= 1u << k;
-                    ++ndup;
-                }
-            }
-        }
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, d);
+        if (int(lane_id()) >= d) inc += y;
     }
-    // 3. duplicates before every tile position; the tile's kept count
-    uint64_t tdup;
-    const uint32_t dex = uint32_t(block_exclusive_scan<uint64_t>(ndup, sh, &tdup));
-    {
+    if (lane_id() == 31) s_wdup[threadIdx.x >> 5] = inc;
+    __syncthreads();
+    uint32_t dex = inc - ndup, tdup = 0;
+#pragma unroll
+    for (int w = 0; w < kThreads / 32; ++w) {
+        const uint32_t x = s_wdup[w];
+        dex += w < int(threadIdx.x >> 5) ? x : 0u;
+        tdup += x;
+    }
+    const uint64_t kept = len - tdup;
+    if (tdup) {  // block-uniform: close the duplicates' gaps (kept items move left)
+        s_tdup[threadIdx.x] = dex;
+        s_dmask[threadIdx.x] = dmask;
+        uint32_t v[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) v[k] = k0 + k < k1 ? s_m[OI(k0 + k)] : 0u;
+        __syncthreads();
         uint32_t run = dex;
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
-            if (k0 + k < k1) s_dpre[k0 + k] = uint16_t(run);
-            run += (dmask >> k) & 1u;
+            const uint32_t pos = k0 + k;
+            if (pos < k1) {
+                if ((dmask >> k) & 1u) ++run;
+                else s_m[OI(pos - run)] = v[k];
+            }
         }
-        if (k1 == len && k0 < k1) s_dpre[len] = uint16_t(run);
     }
-    const uint64_t kept = len - tdup;
     // 4. decoupled look-back over the tiles' kept counts, one warp reading a
-    //    window of 32 predecessors per round trip (a serial one-tile-per-load
-    //    look-back falls behind the tiles in flight and serialises the grid)
+    //    window of 32 x kLB predecessors per round trip (lane l holds the
+    //    l-th group of kLB, nearest first)
+#ifdef SPBLA_EW_FAKE_LB  // timing experiment only: no look-back (wrong offsets)
+    if (threadIdx.x == 0) s_base = d0;
+    if (false) {
+#else
     if (threadIdx.x < 32) {
+#endif
         const unsigned lane = lane_id();
         uint64_t prefix = 0;
         if (t == 0) {
             if (lane == 0) st_relaxed(&status[0], kFlagPre | kept);
         } else {
             if (lane == 0) st_relaxed(&status[t], kFlagAgg | kept);
-            for (long j = long(t) - 1;; j -= 32) {
-                const long idx = j - long(lane);  // lane 0 = the nearest predecessor
-                uint64_t s = idx >= 0 ? ld_relaxed(&status[idx]) : kFlagPre;
-                while (__any_sync(0xffffffffu, (s >> 62) == 0))
-                    if ((s >> 62) == 0) s = ld_relaxed(&status[idx]);
-                const uint32_t pre = __ballot_sync(0xffffffffu, (s >> 62) == 2);
+            for (long j = long(t) - 1;; j -= 32 * kLB) {
+                uint64_t v[kLB];
+#pragma unroll
+                for (int q = 0; q < kLB; ++q) {
+                    const long idx = j - long(lane) * kLB - q;
+                    v[q] = idx >= 0 ? ld_relaxed(&status[idx]) : kFlagPre;
+                }
+                for (;;) {
+                    bool wait = false;
+#pragma unroll
+                    for (int q = 0; q < kLB; ++q) wait |= (v[q] >> 62) == 0;
+                    if (!__any_sync(0xffffffffu, wait)) break;
+                    __nanosleep(32);
+#pragma unroll
+                    for (int q = 0; q < kLB; ++q)
+                        if ((v[q] >> 62) == 0) v[q] = ld_relaxed(&status[j - long(lane) * kLB - q]);
+                }
+                // the lane's sum up to and including its first inclusive prefix
+                int fq = kLB;
+#pragma unroll
+                for (int q = kLB - 1; q >= 0; --q)
+                    if ((v[q] >> 62) == 2) fq = q;
+                uint64_t lsum = 0;
+#pragma unroll
+                for (int q = 0; q < kLB; ++q) lsum += q <= fq ? (v[q] & kValMask) : 0ull;
+                const uint32_t pre = __ballot_sync(0xffffffffu, fq < kLB);
                 const int first = pre ? __ffs(pre) - 1 : 31;
-                prefix += warp_sum(int(lane) <= first ? (s & kValMask) : 0ull);
+                prefix += warp_sum(int(lane) <= first ? lsum : 0ull);
                 if (pre) break;
             }
             if (lane == 0) st_relaxed(&status[t], kFlagPre | (prefix + kept));
         }
         if (lane == 0) s_base = prefix;
     }
-    // 5. kept columns to smem in output order, then coalesced stores
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-        const uint32_t pos = k0 + k;
-        if (pos < k1 && !((dmask >> k) & 1u)) s_out[OI(pos - s_dpre[pos])] = col[k];
-    }
+    // the row offsets' inputs load while warp 0 looks back
+    const uint32_t rlo = tile_rlo[t], rhi = (t + 1 == ntiles) ? m.nrows + 1 : tile_rlo[t + 1];
+    const uint32_t rme = rlo + threadIdx.x;
+    const uint32_t pme = rme < rhi ? uint32_t(P(m, rme) - d0) : 0u;
     __syncthreads();
     const uint64_t base = s_base;
-    for (uint32_t i = threadIdx.x; i < kept; i += kThreads) out[base + i] = s_out[OI(i)];
-    // 6. row offsets of the rows starting in [d0, d1); the last tile also
+    {
+        // 16-B stores: a head of h words brings base + h to a 16-B boundary
+        const uint32_t h = min(uint32_t((4 - (base & 3)) & 3), uint32_t(kept));
+        if (threadIdx.x < h) out[base + threadIdx.x] = s_m[OI(threadIdx.x)];
+        const uint32_t nv = (uint32_t(kept) - h) >> 2;
+        uint4* o4 = reinterpret_cast<uint4*>(out + base + h);
+        for (uint32_t v = threadIdx.x; v < nv; v += kThreads) {
+            const uint32_t i = h + 4 * v;
+            o4[v] = make_uint4(s_m[OI(i)], s_m[OI(i + 1)], s_m[OI(i + 2)], s_m[OI(i + 3)]);
+        }
+        for (uint32_t i = h + 4 * nv + threadIdx.x; i < kept; i += kThreads) out[base + i] = s_m[OI(i)];
+    }
+    // 5. row offsets of the rows starting in [d0, d1); the last tile also
     //    writes the rows starting at L (trailing empty rows, rowptr[nrows])
-    const uint32_t rlo = tile_rlo[t], rhi = (t + 1 == ntiles) ? m.nrows + 1 : tile_rlo[t + 1];
-    for (uint32_t r = rlo + threadIdx.x; r < rhi; r += kThreads) {
-        const uint32_t p = uint32_t(P(m, r) - d0);
-        rowptr[r] = base + p - s_dpre[p];
+    for (uint32_t r = rme; r < rhi; r += kThreads) {
+        const uint32_t p = r == rme ? pme : uint32_t(P(m, r) - d0);
+        uint32_t dpre = tdup;
+        if (p < len) {
+            dpre = 0;
+            if (tdup) {
+                const uint32_t th = p / kItems, j = p % kItems;
+                dpre = s_tdup[th] + __popc(s_dmask[th] & ((1u << j) - 1u));
+            }
+        }
+        rowptr[r] = base + p - dpre;
     }
 }
 

@@ -237,6 +237,39 @@ def test_ewise_add_edge_cases(sp):
     assert_same(X, oracle.ewise_add(OX, OY), "M += N")
 
 
+@pytest.mark.parametrize("kind", ["one_per_row", "long_row_dups", "empty_gaps", "rows_512", "rows_1024"])
+def test_ewise_add_tile_structure(sp, kind):
+    """Merge-path tiles (4096 merged items) whose rows are: more than the
+    1024 staged per tile (one item per row), one row spanning many tiles with
+    duplicates at every tile boundary, thousands of empty rows between rows,
+    and about 512 or 1024 rows per tile (around the staging limit)."""
+    rng = np.random.default_rng(11)
+    if kind == "one_per_row":
+        n, ncols = 30000, 64
+        ra = np.arange(n); ca = rng.integers(0, 4, n)
+        rb = np.arange(0, n, 2); cb = rng.integers(0, 4, len(rb))
+    elif kind == "long_row_dups":
+        n, ncols = 16, 120000
+        ra = np.concatenate([np.full(60000, 3), [0, 15]]); ca = np.concatenate([np.arange(0, 120000, 2), [5, 6]])
+        rb = np.concatenate([np.full(40000, 3), [0, 1]]); cb = np.concatenate([np.arange(0, 120000, 3), [5, 7]])
+    elif kind == "empty_gaps":
+        n, ncols = 400000, 5000
+        rows = rng.choice(n, 300, replace=False)
+        ra = np.repeat(rows, 40); ca = rng.integers(0, ncols, len(ra))
+        rb = np.repeat(rows[::2], 25); cb = rng.integers(0, ncols, len(rb))
+    else:  # 4096 / (na + nb) rows per tile
+        na, nb = (6, 2) if kind == "rows_512" else (3, 1)
+        n, ncols = 12000, 20
+        ra = np.repeat(np.arange(n), na); ca = rng.integers(0, ncols, len(ra))
+        rb = np.repeat(np.arange(n), nb); cb = rng.integers(0, ncols, len(rb))
+    A, OA = both_from_pairs(sp, n, ncols, ra.astype(np.uint32), ca.astype(np.uint32))
+    B, OB = both_from_pairs(sp, n, ncols, rb.astype(np.uint32), cb.astype(np.uint32))
+    want = oracle.ewise_add(OA, OB)
+    assert_same(sp.ewise_add(A, B), want, kind + " A+B")
+    assert_same(sp.ewise_add(B, A), want, kind + " B+A")
+    assert_same(sp.ewise_add(A, A), OA, kind + " A+A")
+
+
 # ------------------------------------------------------------------ Kronecker
 
 def test_kronecker(sp):
