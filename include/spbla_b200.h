@@ -118,6 +118,16 @@ spbla_Status spbla_GetKernelTiming(const char* name, double* total_ms, uint64_t*
  * warp bins W1, W2, W4, W8 (32 E products), hash bins H0..H6; rows above the
  * last go to the bitmap ("dense") bin.  *n: capacity in, count out. */
 spbla_Status spbla_GetEngineThresholds(uint64_t* thresholds, uint32_t* n);
+/* Final step of the row engine (MxM, Build, Transpose, closure steps): the
+ * rows are produced at capacity offsets and then moved to their CSR offsets.
+ * enable != 0 (the default; environment SPBLA_INPLACE_COMPACT=1 starts with
+ * 0): when the device has room for it (free memory >= the result plus
+ * max(2 GB, 1/16 of the device)), the move goes into a new exact-size buffer
+ * -- a plain streaming copy, but the result and the scratch coexist for the
+ * copy; otherwise, and with enable == 0, the move is in place (no second
+ * buffer; tiles ordered by their overlaps, DESIGN.md §4.2 step 5).  Results
+ * are identical either way.  Process-wide; never fails. */
+spbla_Status spbla_SetOutOfPlaceCompaction(int enable);
 
 /* ---- matrix life cycle --------------------------- */
 

@@ -124,6 +124,12 @@ def engine_thresholds():
     return [int(buf[i]) for i in range(n.value)]
 
 
+def set_out_of_place_compaction(enable: bool = True):
+    """spbla_SetOutOfPlaceCompaction: engine compaction into a new buffer when
+    memory allows (results never change)."""
+    _check(_lib().spbla_SetOutOfPlaceCompaction(int(bool(enable))), "spbla_SetOutOfPlaceCompaction")
+
+
 def _ptr(a):
     """Raw address of a torch tensor / numpy array, and whether it is host memory."""
     if a is None:

@@ -32,6 +32,7 @@ SIGNATURES = {
     "spbla_SetKernelTiming": (_int, [_int]),
     "spbla_GetKernelTiming": (_int, [ctypes.c_char_p, ctypes.POINTER(ctypes.c_double), _pu64]),
     "spbla_GetEngineThresholds": (_int, [_pu64, _pu32]),
+    "spbla_SetOutOfPlaceCompaction": (_int, [_int]),
     "spbla_Matrix_New": (_int, [ctypes.POINTER(_vp), _u32, _u32]),
     "spbla_Matrix_Free": (_int, [_vp]),
     "spbla_Matrix_Duplicate": (_int, [_vp, ctypes.POINTER(_vp)]),

@@ -27,6 +27,7 @@ void validate_csr(const off_t64* rowptr, const idx_t* colidx, idx_t nrows, idx_t
 void ktime_enable(bool on);
 void ktime_query(const char* name, double* total_ms, uint64_t* launches);
 void engine_thresholds(uint64_t* out, uint32_t* n);
+void set_out_of_place_compaction(bool on);
 }  // namespace spbla
 
 using namespace spbla;
@@ -188,6 +189,10 @@ spbla_Status spbla_GetEngineThresholds(uint64_t* thresholds, uint32_t* n) {
         NEED(thresholds && n, "null argument");
         engine_thresholds(thresholds, n);
     });
+}
+
+spbla_Status spbla_SetOutOfPlaceCompaction(int enable) {
+    return guarded([&] { set_out_of_place_compaction(enable != 0); });
 }
 void spbla_ResetLaunchCount(void) { ctx().launches = 0; }
 

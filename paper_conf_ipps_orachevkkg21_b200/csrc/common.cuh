@@ -50,6 +50,10 @@ void require_init();
 // with temporaries (a pool miss maps fresh memory: ~60 ms per GB on B200).
 void* dev_alloc(size_t bytes, bool mat = false);
 void dev_free(void* p, size_t bytes);
+// true if dev_alloc(bytes, mat) can be served without evicting the cache: a
+// cached block of its size class, or free device (+ pool) memory with a
+// margin of max(2 GB, 1/16 of the device)
+bool dev_can_alloc(size_t bytes, bool mat);
 // give the size-class cache's blocks back to the pools (Finalize, OOM retry)
 void release_cached_blocks();
 // read `n` uint64 words from device memory (synchronises the stream)

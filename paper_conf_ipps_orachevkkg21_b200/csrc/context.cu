@@ -3,6 +3,7 @@
 // matrix storage helpers.
 #include "common.cuh"
 
+#include <algorithm>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -113,6 +114,24 @@ void* dev_alloc(size_t bytes, bool mat) {
     g_ctx.cur_bytes += bytes;
     if (g_ctx.cur_bytes > g_ctx.peak_bytes) g_ctx.peak_bytes = g_ctx.cur_bytes;
     return p;
+}
+
+bool dev_can_alloc(size_t bytes, bool mat) {
+    require_init();
+    const size_t cb = size_class(bytes);
+    auto it = g_free.find(cb);
+    if (it != g_free.end() && !it->second.empty()) return true;  // a cached block of the class
+    size_t fr = 0, tot = 0;
+    if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return false;
+    }
+    cudaMemPool_t pool = mat ? g_ctx.mat_pool : g_ctx.pool;
+    uint64_t r = 0, u = 0;
+    cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &r);
+    cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &u);
+    const size_t margin = std::max<size_t>(size_t(2) << 30, tot / 16);  // headroom for the rest of the operation
+    return fr + (r > u ? r - u : 0) >= cb + margin;
 }
 
 void dev_free(void* p, size_t bytes) {

@@ -45,20 +45,29 @@ __global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const 
     const unsigned lane = threadIdx.x & 31, g = lane & (kGroup - 1);
     const unsigned gshift = lane & ~(kGroup - 1);  // first lane of this row's group
     const size_t ngroups = (size_t(gridDim.x) * blockDim.x) / kGroup;
-    // warp-uniform loop: every lane of a warp runs the same trip count
-    for (size_t rb = (blockIdx.x * size_t(blockDim.x) + (threadIdx.x & ~31u)) / kGroup; rb < A.nrows;
-         rb += ngroups) {
+    // warp-uniform loop: every lane of a warp runs the same trip count.  The
+    // row offsets of the group's next row are loaded one iteration ahead
+    // (the loop is a chain of dependent loads: offsets, colidx, B records)
+    size_t rb = (blockIdx.x * size_t(blockDim.x) + (threadIdx.x & ~31u)) / kGroup;
+    off_t64 bn = 0, en = 0;
+    if (rb + lane / kGroup < A.nrows) {
+        bn = A.rowptr[rb + lane / kGroup];
+        en = A.rowptr[rb + lane / kGroup + 1];
+    }
+    for (; rb < A.nrows; rb += ngroups) {
         const size_t r = rb + lane / kGroup;
         const bool valid = r < A.nrows;
         uint64_t s = 0;
-        off_t64 b = 0, e = 0;
+        const off_t64 b = valid ? bn : 0, e = valid ? en : 0;
+        if (r + ngroups < A.nrows) {
+            bn = A.rowptr[r + ngroups];
+            en = A.rowptr[r + ngroups + 1];
+        }
         uint32_t cn = 0, cl = 0;  // running non-empty count / product prefix of the row
         uint32_t lcr = 0;         // |C[r]| (accumulate)
         idx_t lo = 0xFFFFFFFFu, hi = 0;
         uint4* drow = nullptr;
         if (valid) {
-            b = A.rowptr[r];
-            e = A.rowptr[r + 1];
             drow = desc + (b + r);  // room for the C[r] segment in front
             if (crp) {
                 const off_t64 cb = crp[r];

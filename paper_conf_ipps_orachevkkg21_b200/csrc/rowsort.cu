@@ -161,15 +161,17 @@ __device__ __forceinline__ uint64_t seg_base(const SegSource& s, idx_t r) {
     return s.kind == 1 ? 0 : s.dbase[r] + r;
 }
 // stage one descriptor as entry i of the batch whose concatenation starts at base
+// (nf: entries of sd_first; a batch with more products than nf << kFirstShift
+// leaves the table partial and the gather binary-searches instead)
 __device__ __forceinline__ void stage_one(const uint4& e, uint32_t i, uint32_t base, const idx_t** sd_ptr,
-                                          uint32_t* sd_end, uint32_t* sd_first) {
+                                          uint32_t* sd_end, uint32_t* sd_first, uint32_t nf = 0xFFFFFFFFu) {
     const idx_t* p = reinterpret_cast<const idx_t*>((uint64_t(e.y) << 32) | e.x);
     const uint32_t end = e.w - base, start = end - e.z;
     sd_ptr[i] = p - start;
     sd_end[i] = end;
     if (sd_first) {
 #pragma unroll 1
-        for (uint32_t j = (start + (1u << kFirstShift) - 1) >> kFirstShift; (j << kFirstShift) < end; ++j)
+        for (uint32_t j = (start + (1u << kFirstShift) - 1) >> kFirstShift; (j << kFirstShift) < end && j < nf; ++j)
             sd_first[j] = i;
     }
 }
@@ -177,7 +179,7 @@ __device__ __forceinline__ void stage_one(const uint4& e, uint32_t i, uint32_t b
 template <int THREADS, int KINDT = -1>
 __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, uint64_t sbase, uint32_t s0,
                                                    uint32_t n, const idx_t** sd_ptr, uint32_t* sd_end,
-                                                   uint32_t* sd_first) {
+                                                   uint32_t* sd_first, uint32_t nf = 0xFFFFFFFFu) {
     if ((KINDT >= 0 ? KINDT : s.kind) == 1) {  // one segment
         if (threadIdx.x == 0) {
             const off_t64 b = s.lrp[r];
@@ -190,7 +192,7 @@ __device__ __forceinline__ uint32_t stage_segments(const SegSource& s, idx_t r, 
     const uint4* d = s.desc + (sbase + s0);
     const uint32_t base = s0 ? s.desc[sbase + s0 - 1].w : 0u;
 #pragma unroll 1
-    for (uint32_t i = threadIdx.x; i < n; i += THREADS) stage_one(d[i], i, base, sd_ptr, sd_end, sd_first);
+    for (uint32_t i = threadIdx.x; i < n; i += THREADS) stage_one(d[i], i, base, sd_ptr, sd_end, sd_first, nf);
     __syncthreads();
     return d[n - 1].w - base;
 }
@@ -210,12 +212,14 @@ template <int THREADS, int U, int KINDT = -1, typename F>
 __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint64_t sbase, uint32_t nseg,
                                                const idx_t** sd_ptr, uint32_t* sd_end, uint32_t* sd_first,
                                                uint32_t batch, bool prestaged, F&& f,
-                                               const volatile uint32_t* abort = nullptr) {
+                                               const volatile uint32_t* abort = nullptr, uint32_t nf = 0xFFFFFFFFu) {
     for (uint32_t s0 = 0; s0 < nseg; s0 += batch) {
         const uint32_t ns = min(batch, nseg - s0);
         const uint32_t total = (s0 == 0 && prestaged)
                                    ? sd_end[ns - 1]
-                                   : stage_segments<THREADS, KINDT>(s, r, sbase, s0, ns, sd_ptr, sd_end, sd_first);
+                                   : stage_segments<THREADS, KINDT>(s, r, sbase, s0, ns, sd_ptr, sd_end, sd_first, nf);
+        // (a partial lookup table: binary search)
+        const uint32_t* sdf = (sd_first && uint64_t(total) <= (uint64_t(nf) << kFirstShift)) ? sd_first : nullptr;
 #ifdef SPBLA_PROBE
         if (threadIdx.x == 0 && s0 == 0) s_probe_ext[3] = gtimer();  // stage done
 #endif
@@ -230,8 +234,8 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
             uint32_t k;
             if ((KINDT >= 0 ? KINDT : s.kind) == 1) {
                 k = 0;
-            } else if (sd_first) {
-                k = sd_first[q0 >> kFirstShift];
+            } else if (sdf) {
+                k = sdf[q0 >> kFirstShift];
                 while (sd_end[k] <= q0) ++k;
             } else {
                 uint32_t lo = 0, hi = ns - 1;  // first segment whose end exceeds q0
@@ -550,6 +554,24 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             if (i < n) stage_one(pfd[k], i, 0u, sd_ptr, sd_end, sd_first);
         }
     };
+    // ... and, once the descriptors have arrived, a bulk-async L2 prefetch of
+    // the B rows they point at (cp.async.bulk.prefetch: one instruction per
+    // segment, 16-B aligned cover), issued before pass B so the next row's
+    // gather finds its first batch in L2
+    auto pf_l2 = [&](const RowPlan& N) {
+        if (!pre || N.mode == kPlanEnd) return;
+        const uint32_t n = min(N.rec.nseg, BATCH);
+#pragma unroll
+        for (int k = 0; k < PF; ++k) {
+            const uint32_t i = threadIdx.x + k * THREADS;
+            if (i < n) {
+                const uint64_t a = (uint64_t(pfd[k].y) << 32) | pfd[k].x;
+                const uint64_t a0 = a & ~uint64_t(15), a1 = (a + 4ull * pfd[k].z + 15) & ~uint64_t(15);
+                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(uint32_t(a1 - a0))
+                             : "memory");
+            }
+        }
+    };
     // the table is kept clean between rows (all slots 0xFFFF, counters 0):
     // every row restores what it dirtied before the end-of-row barrier
 #pragma unroll 1
@@ -812,6 +834,9 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             }
             if (threadIdx.x == 0) counts[r] = carry;
             __syncwarp();
+#ifndef SPBLA_NO_L2PF
+            pf_l2(N);  // (the descriptors were loaded before the overflow pass and the multi-scan)
+#endif
             PROBE(6);
             // ---- pass B: warp-cooperative emission of the warp's own pairs --------
             // (pairs 32w + i*THREADS + j were sorted and scanned by this warp's
@@ -926,15 +951,21 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     }
 }
 
-// ---- 4c. block two-level bitmap bin ------------------------------------------
+// ---- 4c. block bitmap bin ----------------------------------------------------
 // dynamic smem: sd_ptr[BATCH] | sd_end[BATCH] | bm[BITS/32] | top[BITS/1024]
-// top bit t set <=> bm word t may be non-zero.  Emission walks the top level,
-// so clearing and emitting cost O(words touched + BITS/1024).  Two configs:
-// 1024 threads x 1.5 Mi-bit windows, one block per SM (the dense bin: rows
-// with > 40960 products) and 256 threads x 256 Ki-bit windows, 6 blocks per
-// SM (hash-bin rows that fell back - e.g. duplicate-heavy closure rows - and
-// whose span fits two windows).
-template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS, bool FCOUNT>
+// Two configs:
+// * 256 threads x 256 Ki-bit windows, 6 blocks per SM (TOPLVL: hash-bin rows
+//   that fell back - e.g. duplicate-heavy closure rows - and whose span fits
+//   two windows): two levels, top bit t set <=> bm word t may be non-zero;
+//   emission walks the top level, so clearing and emitting cost O(words
+//   touched + BITS/1024) -- those rows are sparse in their window.
+// * 1024 threads x 1.5 Mi-bit windows, one block per SM (the dense bin: rows
+//   with > 40960 products, at least ~1 product per 40 columns of the span):
+//   one level -- the products set bits with non-returning atomics and the
+//   emission walks the window's words directly (a count pass and an emit
+//   pass); the top-level words serve as the gather's segment lookup table
+//   (sd_first) instead.
+template <int THREADS, uint32_t BATCH, int FLATU, uint32_t BITS, bool FCOUNT, bool TOPLVL>
 __global__ void __launch_bounds__(THREADS)
 dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ bounds,
                  const uint2* __restrict__ range, idx_t ncols, idx_t* __restrict__ scratch,
@@ -947,6 +978,8 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
     uint32_t* sd_end = reinterpret_cast<uint32_t*>(smem_raw + BATCH * sizeof(void*));
     uint32_t* bm = reinterpret_cast<uint32_t*>(smem_raw + BATCH * (sizeof(void*) + sizeof(uint32_t)));
     uint32_t* top = bm + kWords;
+    uint32_t* sd_first = TOPLVL ? nullptr : top;  // (one level: the top words hold the segment lookup table)
+    static_assert(!FCOUNT || TOPLVL, "the gather-time count needs the top level");
     __shared__ uint32_t s_w[33];
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     fill_words(bm, kWords + kTop, 0u, THREADS);  // kept clean between rows
@@ -1041,9 +1074,13 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                 if (c >= wlo && c < whi) {
                     const uint32_t d = uint32_t(c - wlo);
                     const uint32_t bit = 1u << (d & 31);
-                    const uint32_t old = atomicOr(&bm[d >> 5], bit);
-                    if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
-                    if (FCOUNT && !(old & bit)) atomicAdd(&s_w[(d >> 10) / tcw], 1u);
+                    if (TOPLVL) {
+                        const uint32_t old = atomicOr(&bm[d >> 5], bit);
+                        if (old == 0) atomicOr(&top[d >> 10], 1u << ((d >> 5) & 31));
+                        if (FCOUNT && !(old & bit)) atomicAdd(&s_w[(d >> 10) / tcw], 1u);
+                    } else {
+                        atomicOr(&bm[d >> 5], bit);  // (result unused: no wait on the atomic)
+                    }
                 }
             };
             if (part) {  // this window's slice: coalesced reads of the scattered products
@@ -1051,42 +1088,31 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                 for (uint32_t i = sb + threadIdx.x; i < se; i += THREADS) set_bit(out[i]);
                 __syncthreads();
             } else {
-                block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, nullptr, BATCH,
-                                               false, set_bit);
+                block_products<THREADS, FLATU>(src, r, seg_base(src, r), num_segs(src, r), sd_ptr, sd_end, sd_first, BATCH,
+                                               false, set_bit, nullptr, kTop);
             }
-            // emission over the top level: warp w owns top words [tb, te),
-            // read 32 at a time (one per lane); a ballot gives the non-zero
-            // ones and the warp visits only those (rows of a few hundred
-            // columns leave most top words empty: the per-word loop was the
-            // kernel's largest instruction count)
-            if (!FCOUNT) {  // (FCOUNT: the gather ended with a barrier after the counts)
+            if (!TOPLVL) {
+                // one level: warp w owns the words [wb, we) of the window
+                // (32 top-word spans); a count pass, a scan, an emit pass that
+                // also clears the words
+                const uint32_t nwd = uint32_t((whi - wlo + 31) >> 5);
+                const uint32_t wb = min(nwd, tb * 32), we = min(nwd, te * 32);
                 uint32_t cnt = 0;
-                for (uint32_t t0 = tb; t0 < te; t0 += 32) {
-                    const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
-                    for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {  // warp-uniform
-                        const uint32_t j = __ffs(m) - 1, t = t0 + j;
-                        const uint32_t tw = __shfl_sync(FULL, tl, j);
-                        const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
-                        cnt += __popc(word);
-                    }
-                }
+                for (uint32_t i = wb + lane; i < we; i += 32) cnt += __popc(bm[i]);
                 cnt = warp_sum(cnt);
                 if (lane == 0) s_w[wib] = cnt;
                 __syncthreads();
-            }
-            scan_warp_counts<NW>(s_w);
-            uint32_t pos = s_w[wib];
-            for (uint32_t t0 = tb; t0 < te; t0 += 32) {
-                const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
-                for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {
-                    const uint32_t j = __ffs(m) - 1, t = t0 + j;
-                    const uint32_t tw = __shfl_sync(FULL, tl, j);
-                    uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
-                    if ((tw >> lane) & 1u) bm[t * 32 + lane] = 0u;  // clean for the next row/window
+                scan_warp_counts<NW>(s_w);
+                uint32_t pos = s_w[wib];
+                for (uint32_t i0 = wb; i0 < we; i0 += 32) {
+                    const uint32_t i = i0 + lane;
+                    uint32_t word = i < we ? bm[i] : 0u;
+                    if (!__any_sync(FULL, word != 0)) continue;  // warp-uniform
+                    if (word) bm[i] = 0u;  // clean for the next row/window
                     const uint32_t c = __popc(word);
                     const uint32_t inc = warp_inclusive_scan(c);
                     uint32_t o = pos + inc - c;
-                    const uint64_t colbase = wlo + (uint64_t(t * 32 + lane) << 5);
+                    const uint64_t colbase = wlo + (uint64_t(i) << 5);
                     while (word) {
                         const int bit = __ffs(word) - 1;
                         word &= word - 1;
@@ -1094,7 +1120,49 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
                     }
                     pos += __shfl_sync(FULL, inc, 31);
                 }
-                if (tl) top[t0 + lane] = 0u;  // (each lane its own top word; tw came by shuffle)
+            } else {
+                // emission over the top level: warp w owns top words [tb, te),
+                // read 32 at a time (one per lane); a ballot gives the non-zero
+                // ones and the warp visits only those (rows of a few hundred
+                // columns leave most top words empty: the per-word loop was the
+                // kernel's largest instruction count)
+                if (!FCOUNT) {  // (FCOUNT: the gather ended with a barrier after the counts)
+                    uint32_t cnt = 0;
+                    for (uint32_t t0 = tb; t0 < te; t0 += 32) {
+                        const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
+                        for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {  // warp-uniform
+                            const uint32_t j = __ffs(m) - 1, t = t0 + j;
+                            const uint32_t tw = __shfl_sync(FULL, tl, j);
+                            const uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                            cnt += __popc(word);
+                        }
+                    }
+                    cnt = warp_sum(cnt);
+                    if (lane == 0) s_w[wib] = cnt;
+                    __syncthreads();
+                }
+                scan_warp_counts<NW>(s_w);
+                uint32_t pos = s_w[wib];
+                for (uint32_t t0 = tb; t0 < te; t0 += 32) {
+                    const uint32_t tl = t0 + lane < te ? top[t0 + lane] : 0u;
+                    for (uint32_t m = __ballot_sync(FULL, tl != 0); m; m &= m - 1) {
+                        const uint32_t j = __ffs(m) - 1, t = t0 + j;
+                        const uint32_t tw = __shfl_sync(FULL, tl, j);
+                        uint32_t word = (tw >> lane) & 1u ? bm[t * 32 + lane] : 0u;
+                        if ((tw >> lane) & 1u) bm[t * 32 + lane] = 0u;  // clean for the next row/window
+                        const uint32_t c = __popc(word);
+                        const uint32_t inc = warp_inclusive_scan(c);
+                        uint32_t o = pos + inc - c;
+                        const uint64_t colbase = wlo + (uint64_t(t * 32 + lane) << 5);
+                        while (word) {
+                            const int bit = __ffs(word) - 1;
+                            word &= word - 1;
+                            out[written + o++] = idx_t(colbase + bit);
+                        }
+                        pos += __shfl_sync(FULL, inc, 31);
+                    }
+                    if (tl) top[t0 + lane] = 0u;  // (each lane its own top word; tw came by shuffle)
+                }
             }
             written += s_w[32];
             __syncthreads();
@@ -1401,8 +1469,12 @@ __global__ void tile_deps_kernel(const uint64_t* __restrict__ src_lo, uint64_t n
     }
 }
 
+// INPLACE = false: the same tile copy from the scratch buf into a separate
+// exact-size buffer dst (no read/write ordering between tiles: a plain
+// streaming copy)
+template <bool INPLACE>
 __global__ void __launch_bounds__(kCThreads, kCMinB)
-compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint64_t* __restrict__ rowptr,
+compact_inplace_kernel(idx_t* buf, idx_t* dst, const uint64_t* __restrict__ soff, const uint64_t* __restrict__ rowptr,
                        const uint32_t* __restrict__ tile_row, const uint2* __restrict__ wait_range,
                        idx_t nrows, uint64_t nnz, uint32_t* flags, uint32_t* ticket) {
     // staged rows of the tile in tile-local coordinates: s_beg[i] = start of
@@ -1421,7 +1493,7 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
                 // rows holding d0 and (a bound on the row holding) d1-1
                 s_r0 = tile_row[t];
                 s_r1 = tile_row[t + 1];
-                s_w = wait_range[t];
+                if (INPLACE) s_w = wait_range[t];
             }
         }
         __syncthreads();
@@ -1431,7 +1503,7 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
         const uint32_t n = uint32_t(min(uint64_t(kCT), nnz - d0));  // tile length
         const uint32_t r0 = s_r0, r1 = s_r1;
         const uint64_t slack1 = soff[r1] - rowptr[r1];
-        if (slack1 == 0) {  // whole tile already in place (slack is nondecreasing)
+        if (INPLACE && slack1 == 0) {  // whole tile already in place (slack is nondecreasing)
             if (threadIdx.x == 0) st_release_u32(&flags[t], 1u);
             __syncthreads();
             continue;
@@ -1495,18 +1567,20 @@ compact_inplace_kernel(idx_t* buf, const uint64_t* __restrict__ soff, const uint
                     }
                 }
         }
-        // publish "read done": the barrier orders every thread's loads before
-        // thread 0's gpu-scope fence and release store
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            __threadfence();
-            st_release_u32(&flags[t], 1u);
+        if (INPLACE) {
+            // publish "read done": the barrier orders every thread's loads before
+            // thread 0's gpu-scope fence and release store
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                __threadfence();
+                st_release_u32(&flags[t], 1u);
+            }
+            // wait for the earlier tiles that read sources inside [d0, d1)
+            for (uint32_t j = s_w.x + threadIdx.x; j < s_w.y; j += kCThreads)
+                while (ld_acquire_u32(&flags[j]) == 0) __nanosleep(64);
         }
-        // wait for the earlier tiles that read sources inside [d0, d1)
-        for (uint32_t j = s_w.x + threadIdx.x; j < s_w.y; j += kCThreads)
-            while (ld_acquire_u32(&flags[j]) == 0) __nanosleep(64);
         __syncthreads();
-        idx_t* dp = buf + d0;  // 16-B aligned (kCT and the buffer are)
+        idx_t* dp = (INPLACE ? buf : dst) + d0;  // 16-B aligned (kCT and the buffers are)
 #pragma unroll
         for (int k = 0; k < kCChunks; ++k) {
             const uint32_t e0 = 4 * (k * kCThreads + threadIdx.x);
@@ -1589,12 +1663,12 @@ HBIN(H6, H6_CFG)
 constexpr size_t kDSmem = kDBatch * kSegBytes + (kDenseBits / 32 + kDenseBits / 1024) * sizeof(uint32_t);
 static_assert(kDSmem + 2048 <= 227 * 1024, "dense bin smem");
 static_assert((kDenseBits / 1024) % 32 == 0, "dense bin: top words per warp");
-#define DENSE dense_bin_kernel<1024, kDBatch, 8, kDenseBits, false>
+#define DENSE dense_bin_kernel<1024, kDBatch, 8, kDenseBits, false, false>
 constexpr uint32_t kSDenseBits = 1u << 18, kSDBatch = 192;
 constexpr int kSDPerSM = 6;  // blocks per SM (the kernel is barrier/latency-bound: residency pays)
 constexpr size_t kSDSmem = kSDBatch * kSegBytes + (kSDenseBits / 32 + kSDenseBits / 1024) * sizeof(uint32_t);
 static_assert(kSDPerSM * (kSDSmem + 1024 + 512) <= 228 * 1024, "small dense bin residency");
-#define SDENSE dense_bin_kernel<256, kSDBatch, 4, kSDenseBits, true>
+#define SDENSE dense_bin_kernel<256, kSDBatch, 4, kSDenseBits, true, true>
 
 static void ensure_attrs() {
     static int done_dev = -1;
@@ -1617,6 +1691,9 @@ static void ensure_attrs() {
     CUDA_CHECK(cudaFuncSetAttribute(SDENSE, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kSDSmem)));
     done_dev = ctx().device;
 }
+
+// out-of-place compaction allowed (spbla_SetCompactionMode; env SPBLA_INPLACE_COMPACT=1 turns it off)
+static bool g_oop_compact = std::getenv("SPBLA_INPLACE_COMPACT") == nullptr;
 
 void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* ub, const uint2* range,
                 Matrix* out) {
@@ -1760,27 +1837,38 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     const uint64_t nnz = h[0];
     ovf_rows.release();
     counts.release();
-    // 6. compaction: in place when the capacity slack is small (the result
-    //    keeps the buffer, colidx_cap >= nnz), else into an exact buffer
-    const bool inplace = scratch_total - nnz <= scratch_total / 8;
+    // 6. compaction: when the capacity slack is small, a tile copy -- into a
+    //    separate exact-size buffer when the device has room for it (a plain
+    //    streaming copy), else in place (tiles ordered by their read/write
+    //    overlaps; the result keeps the scratch buffer, colidx_cap >= nnz);
+    //    a large slack is copied row by row into an exact buffer
+    const bool small_slack = scratch_total - nnz <= scratch_total / 8;
     DevBuf<idx_t> colidx;
-    if (nnz && inplace) {
+    bool inplace = false;
+    if (nnz && small_slack) {
         const uint64_t ntiles = ceil_div(nnz, kCT);
+        inplace = !(g_oop_compact && dev_can_alloc(nnz * sizeof(idx_t), kMat));
+        if (!inplace) colidx.alloc(nnz, kMat);
         // flags[ntiles] | ticket | tile_row[ntiles + 1]; src_lo[ntiles]; wait_range[ntiles]
         DevBuf<uint32_t> flags(2 * ntiles + 2);
         DevBuf<uint64_t> src_lo(ntiles);
-        DevBuf<uint2> wait_range(ntiles);
+        DevBuf<uint2> wait_range(inplace ? ntiles : 0);
         uint32_t* tile_row = flags.p + ntiles + 1;
         memset_async(flags.p, 0, (ntiles + 1) * sizeof(uint32_t));
         t = ktime_begin("compact", st);
         tile_rows_kernel<<<gb, 256, 0, st>>>(rowptr.p, soff.p, nrows, ntiles, tile_row, src_lo.p);
-        tile_deps_kernel<<<(unsigned)std::min<uint64_t>(ceil_div(ntiles, 256), uint64_t(nsm) * 8), 256, 0, st>>>(
-            src_lo.p, ntiles, nnz, wait_range.p);
-        compact_inplace_kernel<<<nsm * kCMinB * 2, kCThreads, 0, st>>>(scratch.p, soff.p, rowptr.p, tile_row, wait_range.p,
-                                                             nrows, nnz, flags.p, flags.p + ntiles);
-        count_launch(2);
+        if (inplace) {
+            tile_deps_kernel<<<(unsigned)std::min<uint64_t>(ceil_div(ntiles, 256), uint64_t(nsm) * 8), 256, 0, st>>>(
+                src_lo.p, ntiles, nnz, wait_range.p);
+            compact_inplace_kernel<true><<<nsm * kCMinB * 2, kCThreads, 0, st>>>(
+                scratch.p, nullptr, soff.p, rowptr.p, tile_row, wait_range.p, nrows, nnz, flags.p, flags.p + ntiles);
+            count_launch(3);
+        } else {
+            compact_inplace_kernel<false><<<nsm * kCMinB * 2, kCThreads, 0, st>>>(
+                scratch.p, colidx.p, soff.p, rowptr.p, tile_row, nullptr, nrows, nnz, flags.p, flags.p + ntiles);
+            count_launch(2);
+        }
         ktime_end(t);
-        count_launch();
         check_launch("compact_inplace_kernel");
     } else if (nnz) {
         colidx.alloc(nnz, kMat);
@@ -1801,6 +1889,8 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
         matrix_replace(out, rowptr.detach(), rcap, colidx.detach(), ccap, nnz);
     }
 }
+
+void set_out_of_place_compaction(bool on) { g_oop_compact = on; }
 
 void engine_thresholds(uint64_t* out, uint32_t* n) {
     // ub upper limits of bins W1, W2, W4, W8, H0..H6 (DENSE above)

@@ -57,6 +57,30 @@ def test_build_inplace_compaction(sp, nrows, per_row, ncols, dup_every):
     assert_same(M, O, "build in-place compaction")
 
 
+@pytest.mark.parametrize("oop", [False, True], ids=["in_place", "out_of_place"])
+def test_compaction_modes(sp, oop):
+    """spbla_SetOutOfPlaceCompaction: the engine's final move into CSR in place
+    (tiles ordered by their overlaps) and into a new exact buffer give the
+    same CSR (Build with a small slack over many tiles, A.A, C += A.A)."""
+    sp.set_out_of_place_compaction(oop)
+    try:
+        rng = np.random.default_rng(9)
+        nrows, per_row = 1 << 18, 6
+        r = np.repeat(np.arange(nrows, dtype=np.uint32), per_row)
+        c = rng.integers(0, 1 << 20, len(r)).astype(np.uint32)
+        M, O = both_from_pairs(sp, nrows, 1 << 20, r[::-1].copy(), c)
+        assert_same(M, O, "build")
+        rr, cc = spgen.rmat_pairs(12, 16, 0.45, 0.22, 0.22, seed=11)
+        A, OA = both_from_pairs(sp, 4096, 4096, rr, cc)
+        assert_same(sp.mxm(A, A), oracle.mxm(OA, OA), "A.A")
+        r2, c2 = spgen.uniform_pairs(4096, 4096, 3, seed=22)
+        C, OC = both_from_pairs(sp, 4096, 4096, r2, c2)
+        sp.MxM(C, A, A, accumulate=True)
+        assert_same(C, oracle.mxm(OA, OA, OC), "C += A.A")
+    finally:
+        sp.set_out_of_place_compaction(True)
+
+
 def test_build_empty_and_errors(sp):
     M = sp.Matrix.new(10, 10)
     M.build(np.zeros(0, np.uint32), np.zeros(0, np.uint32))
@@ -287,6 +311,19 @@ def test_kronecker(sp):
     Z = sp.Matrix.new(3, 5)
     K = sp.kronecker(G, Z)
     assert K.nvals == 0 and K.shape == (256 * 3, 256 * 5)
+
+
+@pytest.mark.parametrize("mb,nb,nvb", [(64, 64, 20), (2048, 100, 8192), (2049, 50, 3000), (4096, 4096, 16384)])
+def test_kronecker_b_sizes(sp, mb, nb, nvb):
+    """Both Kronecker kernels: B staged in shared memory (<= 2048 rows and
+    <= 8192 entries; B with empty rows, B at both limits) and the general
+    kernel (B over either limit); A with empty rows."""
+    ra, ca = spgen.random_pairs(40, 30, 90, seed=mb)
+    A, OA = both_from_pairs(sp, 40, 30, ra, ca)
+    rb, cb = spgen.random_pairs(mb, nb, nvb, seed=nb)
+    B, OB = both_from_pairs(sp, mb, nb, rb, cb)
+    assert_same(sp.kronecker(A, B), oracle.kronecker(OA, OB), f"A(x)B {mb}x{nb}")
+    assert_same(sp.kronecker(B, A), oracle.kronecker(OB, OA), f"B(x)A {mb}x{nb}")
 
 
 # ------------------------------------------------------------------ transpose / reduce / submatrix

@@ -2,7 +2,7 @@
 # Quick GPU iteration: parity tests + bench (both R-MAT workloads) with per-kernel times.
 cd "$(dirname "$0")/.."
 O=gpurun_out/${QDIR:-quick}; mkdir -p $O
-timeout 600 python -m pytest tests -m gpu -x -q --timeout 120 ${PYTEST_K:+-k "$PYTEST_K"} > $O/pytest.txt 2>&1; tail -2 $O/pytest.txt
+timeout 1200 python -m pytest tests -m gpu -x -q --timeout 400 ${PYTEST_K:+-k "$PYTEST_K"} > $O/pytest.txt 2>&1; tail -2 $O/pytest.txt
 for wl in ${WLS:-rmat22_ef32 rmat20_ef16}; do
   timeout 300 python bench.py --workload $wl --no-cpu-baseline --no-e2e --steps 3 > $O/bench_$wl.json 2> $O/bench_$wl.err
   python -c "
