@@ -556,7 +556,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     };
     // ... and, once the descriptors have arrived, a bulk-async L2 prefetch of
     // the B rows they point at (cp.async.bulk.prefetch: one instruction per
-    // segment, 16-B aligned cover), issued before pass B so the next row's
+    // segment), issued before pass B so the next row's
     // gather finds its first batch in L2
     auto pf_l2 = [&](const RowPlan& N) {
         if (!pre || N.mode == kPlanEnd) return;
@@ -566,9 +566,12 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
             const uint32_t i = threadIdx.x + k * THREADS;
             if (i < n) {
                 const uint64_t a = (uint64_t(pfd[k].y) << 32) | pfd[k].x;
-                const uint64_t a0 = a & ~uint64_t(15), a1 = (a + 4ull * pfd[k].z + 15) & ~uint64_t(15);
-                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(uint32_t(a1 - a0))
-                             : "memory");
+                // (16-B aligned inside the segment's allocation: rounded
+                // down at both ends, a tail of < 16 B is not prefetched)
+                const uint64_t a0 = a & ~uint64_t(15), a1 = (a + 4ull * pfd[k].z) & ~uint64_t(15);
+                if (a1 > a0)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(uint32_t(a1 - a0))
+                                 : "memory");
             }
         }
     };
