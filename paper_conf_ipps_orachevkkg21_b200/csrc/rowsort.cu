@@ -28,7 +28,6 @@
 #include "common.cuh"
 
 #include <algorithm>
-#include <cuda/atomic>
 #include <cstdlib>
 
 namespace spbla {
@@ -226,11 +225,16 @@ __device__ __forceinline__ void block_products(const SegSource& s, idx_t r, uint
         for (uint32_t q0 = threadIdx.x * U; q0 < total; q0 += THREADS * U) {
             // a row already bound for the fallback stops gathering (per
             // thread: no barrier inside this loop)
-            // (a relaxed atomic load -- an ordinary LDS -- : the flag is set
-            // concurrently, by atomicExch, from inserting threads)
-            if (abort && cuda::atomic_ref<uint32_t, cuda::thread_scope_block>(*const_cast<uint32_t*>(abort))
-                             .load(cuda::memory_order_relaxed))
-                break;
+            // (a volatile shared load -- LDS -- : the flag is set concurrently,
+            // by atomicExch, from inserting threads; a cuda::atomic_ref load
+            // compiled to a generic strong load)
+            if (abort) {
+                uint32_t fl;
+                asm volatile("ld.volatile.shared.u32 %0, [%1];"
+                             : "=r"(fl)
+                             : "r"(uint32_t(__cvta_generic_to_shared(const_cast<uint32_t*>(abort)))));
+                if (fl) break;
+            }
             uint32_t k;
             if ((KINDT >= 0 ? KINDT : s.kind) == 1) {
                 k = 0;
