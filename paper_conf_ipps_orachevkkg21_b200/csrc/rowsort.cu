@@ -1585,8 +1585,9 @@ compact_inplace_kernel(idx_t* buf, idx_t* dst, const uint64_t* __restrict__ soff
             // wait for the earlier tiles that read sources inside [d0, d1)
             for (uint32_t j = s_w.x + threadIdx.x; j < s_w.y; j += kCThreads)
                 while (ld_acquire_u32(&flags[j]) == 0) __nanosleep(64);
+            __syncthreads();
         }
-        __syncthreads();
+        // (out of place: each thread stores what it loaded, no barrier)
         idx_t* dp = (INPLACE ? buf : dst) + d0;  // 16-B aligned (kCT and the buffers are)
 #pragma unroll
         for (int k = 0; k < kCChunks; ++k) {
