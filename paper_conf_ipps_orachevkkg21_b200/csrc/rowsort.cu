@@ -11,12 +11,13 @@
 //   3. bin_scatter : row lists per bin; make_recs: 40-B work records of the
 //                    hash-bin rows
 //   4. per-bin kernels (heaviest first, persistent grids):
-//        dense (ub > 40960): two-level smem bitmap over 1.5 Mi-column
-//            windows, one 1024-thread block per row; a span of more than
-//            three windows is partitioned by window first (two gathers)
-//        dense_ovf: the same kernel with 256 Ki-column windows for rows the
-//            producer flagged duplicate-heavy (closure steps) and for
-//            hash-bin rows that fell back
+//        dense (ub > 40960): one-level smem bitmap over 1.5 Mi-column
+//            windows (non-returning atomics, word-walk emission), one
+//            1024-thread block per row; a span of more than three windows
+//            is partitioned by window first (two gathers)
+//        dense_ovf: the same kernel with 256 Ki-column windows and a
+//            two-level bitmap for rows the producer flagged duplicate-heavy
+//            (closure steps) and for hash-bin rows that fell back
 //        hash H6..H0 (ub <= 40960 .. 512): bucketed order-preserving hash in
 //            smem (bucket = floor((c - lo) / W), 16 slots of 16-bit offsets,
 //            one atomicAdd per insert), 16x2 SIMD Batcher sort per bucket
@@ -24,7 +25,9 @@
 //            span is small
 //        warp W8..W1 (ub <= 256): one warp per row, register bitonic sort
 //   5. scan(counts): CSR row offsets
-//   6. compact     : in-place move from capacity offsets to CSR offsets
+//   6. compact     : move from capacity offsets to CSR offsets -- a tile copy
+//                    into a new exact buffer when memory allows, else in
+//                    place (tiles ordered by their overlaps)
 #include "common.cuh"
 
 #include <algorithm>
