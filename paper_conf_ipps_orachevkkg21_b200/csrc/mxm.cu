@@ -36,8 +36,11 @@ __global__ void row_span_kernel(CsrView B, uint2* __restrict__ bspan) {
     }
 }
 
+#ifndef SPBLA_UB_MINB
+#define SPBLA_UB_MINB 1
+#endif
 template <bool INFO>
-__global__ void mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
+__global__ void __launch_bounds__(256, SPBLA_UB_MINB) mxm_ub_kernel(CsrView A, const off_t64* __restrict__ brp, const idx_t* __restrict__ bci,
                               const uint2* __restrict__ bspan, const uint4* __restrict__ binfo,
                               const off_t64* __restrict__ crp,
                               const idx_t* __restrict__ cci, uint64_t* __restrict__ ub, uint2* __restrict__ range,
