@@ -553,18 +553,19 @@ def main():
     if not args.no_e2e:
         # (the device-timed result is no longer needed: its storage goes back
         # to the pools, so the e2e steps run with the same memory headroom)
+        c_rows = C.nrows
         C.free()
         rp_h = torch.empty(A.nrows + 1, dtype=torch.int64).pin_memory()
         ci_h = torch.empty(max(nnzA, 1), dtype=torch.int32).pin_memory()
         A.export_csr(rp_h, ci_h[:nnzA])
-        crp_h = torch.empty(C.nrows + 1, dtype=torch.int64).pin_memory()
+        crp_h = torch.empty(c_rows + 1, dtype=torch.int64).pin_memory()
         cci_h = torch.empty(max(nnzC_local, 1), dtype=torch.int32).pin_memory()
         Ae = sp.Matrix.new(A.nrows, n)
-        Ce = sp.Matrix.new(C.nrows, n)
+        Ce = sp.Matrix.new(c_rows, n)
         e2e_steps = min(args.steps, 3)
         e2e_ms = []
         h2d = (A.nrows + 1) * 8 + nnzA * 4
-        d2h = (C.nrows + 1) * 8 + nnzC_local * 4
+        d2h = (c_rows + 1) * 8 + nnzC_local * 4
         for i in range(e2e_steps + 2):  # (two untimed steps: the pools' blocks reach their steady state)
             if world > 1:
                 dist.barrier()
