@@ -270,7 +270,10 @@ void swap_storage(Matrix* a, Matrix* b) { std::swap(*a, *b); }
 // the last step added less than 1/kSemiNaiveDiv of the entries (|Delta| is
 // known from the nnz read-backs), typically the final confirming step; the
 // iterates and the iteration count are those of the plain loop.
-constexpr uint64_t kSemiNaiveDiv = 8;
+#ifndef SPBLA_SEMI_DIV  // (overridable for a sweep)
+#define SPBLA_SEMI_DIV 8
+#endif
+constexpr uint64_t kSemiNaiveDiv = SPBLA_SEMI_DIV;
 
 // The loop after the first step: prev = C_{k-1}, C = C_k, with
 // C_{k-1} C_{k-1} inside C_k; plain squaring or the semi-naive step
