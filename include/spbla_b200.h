@@ -179,6 +179,15 @@ spbla_Status spbla_Matrix_DevicePointers(spbla_Matrix matrix, const spbla_Offset
  * Errors: null matrix / rowptr, null colidx for a non-empty matrix. */
 spbla_Status spbla_Matrix_ExportRowBlock(spbla_Matrix matrix, spbla_Offset* rowptr, spbla_Index* colidx,
                                         spbla_Offset offset);
+/* spbla_Matrix_ExportRowBlock into ndst destination pairs (rowptrs[k],
+ * colidxs[k]) with one kernel that loads the block once and stores it ndst
+ * times -- the push all-gather over peer memory: the
+ * destinations are every rank's slice of its gathered buffers, mapped into
+ * this process by CUDA IPC, so on an NVSwitch box the stores go over NVLink.
+ * Asynchronous on the library stream; the caller synchronises before the
+ * destination owners read.  Errors: null matrix, null arrays or entries. */
+spbla_Status spbla_Matrix_ExportRowBlockMulti(spbla_Matrix matrix, spbla_Offset* const* rowptrs,
+                                             spbla_Index* const* colidxs, uint32_t ndst, spbla_Offset offset);
 /* Concatenate row blocks (block b: nrows[b] rows, device arrays rowptr[b]
  * starting at 0 and colidx[b] with nnz[b] values) into `matrix` (replaced;
  * its ncols is kept; sum nrows[b] must equal its nrows).  Used to assemble a

@@ -329,6 +329,17 @@ class Matrix:
         _check(_lib().spbla_Matrix_ExportRowBlock(self._h, rowptr.data_ptr(), colidx.data_ptr() if n else None,
                                                   int(offset)), "spbla_Matrix_ExportRowBlock")
 
+    def export_row_block_multi(self, dsts, offset: int):
+        """export_row_block into several (rowptr, colidx) device tensor pairs
+        with one kernel (spbla_Matrix_ExportRowBlockMulti; peer-mapped
+        tensors of other ranks included)."""
+        nd = len(dsts)
+        n = self.nvals
+        rps = (ctypes.c_void_p * max(nd, 1))(*[t.data_ptr() for t, _ in dsts])
+        cis = (ctypes.c_void_p * max(nd, 1))(*[(c.data_ptr() if n else 0) for _, c in dsts])
+        _check(_lib().spbla_Matrix_ExportRowBlockMulti(self._h, rps, cis, nd, int(offset)),
+               "spbla_Matrix_ExportRowBlockMulti")
+
     def assemble_row_blocks(self, blocks):
         """Replace content by the concatenation of row blocks
         [(nrows_b, rowptr_b tensor, colidx_b tensor, nnz_b), ...] (device)."""

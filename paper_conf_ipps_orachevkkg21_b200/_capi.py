@@ -46,6 +46,7 @@ SIGNATURES = {
     "spbla_Matrix_Wrap": (_int, [ctypes.POINTER(_vp), _u32, _u32, _vp, _vp, _u64, _u32]),
     "spbla_Matrix_DevicePointers": (_int, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp)]),
     "spbla_Matrix_ExportRowBlock": (_int, [_vp, _vp, _vp, _u64]),
+    "spbla_Matrix_ExportRowBlockMulti": (_int, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _u32, _u64]),
     "spbla_Matrix_AssembleRowBlocks": (_int, [_vp, _u32, _pu32, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _pu64]),
     "spbla_MxM": (_int, [_vp, _vp, _vp, _u32]),
     "spbla_Matrix_EWiseAdd": (_int, [_vp, _vp, _vp, _u32]),

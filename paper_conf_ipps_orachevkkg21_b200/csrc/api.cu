@@ -19,6 +19,8 @@ void matrix_build(Matrix* m, const idx_t* rows, const idx_t* cols, uint64_t n, u
 void matrix_extract_pairs(const Matrix* m, idx_t* rows, idx_t* cols, uint32_t hints);
 void matrix_export(const Matrix* m, off_t64* rowptr, idx_t* colidx, uint32_t hints);
 void matrix_export_block(const Matrix* m, off_t64* rowptr_out, idx_t* colidx_out, off_t64 offset);
+void matrix_export_block_multi(const Matrix* m, off_t64* const* rowptr_out, idx_t* const* colidx_out, uint32_t ndst,
+                               off_t64 offset);
 void matrix_import(Matrix* m, const off_t64* rowptr, const idx_t* colidx, uint64_t nnz, uint32_t hints);
 void matrix_duplicate(const Matrix* m, Matrix* d);
 void matrix_assemble(Matrix* m, uint32_t nblocks, const idx_t* nrows, const off_t64* const* rowptr,
@@ -287,6 +289,16 @@ spbla_Status spbla_Matrix_ExportRowBlock(spbla_Matrix m, spbla_Offset* rowptr, s
         NEED(m && rowptr, "null argument");
         NEED(m->nnz == 0 || colidx, "null colidx buffer");
         matrix_export_block(m, rowptr, colidx, offset);
+    });
+}
+
+spbla_Status spbla_Matrix_ExportRowBlockMulti(spbla_Matrix m, spbla_Offset* const* rowptrs, spbla_Index* const* colidxs,
+                                             uint32_t ndst, spbla_Offset offset) {
+    return guarded([&] {
+        require_init();
+        NEED(m && (ndst == 0 || (rowptrs && colidxs)), "null argument");
+        for (uint32_t k = 0; k < ndst; ++k) NEED(rowptrs[k] && (m->nnz == 0 || colidxs[k]), "null destination");
+        if (ndst) matrix_export_block_multi(m, rowptrs, colidxs, ndst, offset);
     });
 }
 

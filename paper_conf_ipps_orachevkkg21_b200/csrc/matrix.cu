@@ -82,6 +82,29 @@ __global__ void shift_rowptr_kernel(const off_t64* __restrict__ in, idx_t n, off
 
 __global__ void set_word_kernel(off_t64* p, off_t64 v) { *p = v; }
 
+// One row block pushed to up to kMaxPeerDst destinations at once (the
+// all-gather over peer memory): every element is loaded once
+// and stored to each destination -- on an NVSwitch box the destinations are
+// the other GPUs' gathered buffers, mapped into this process (CUDA IPC), so
+// the stores travel over NVLink.  Warps store contiguous 128-B runs.
+constexpr uint32_t kMaxPeerDst = 8;
+struct PeerDst {
+    off_t64* rp[kMaxPeerDst];
+    idx_t* ci[kMaxPeerDst];
+};
+__global__ void export_multi_kernel(const off_t64* __restrict__ rp, idx_t nrows, const idx_t* __restrict__ ci,
+                                    uint64_t nnz, off_t64 add, PeerDst d, uint32_t ndst) {
+    const size_t stride = size_t(gridDim.x) * blockDim.x;
+    for (size_t i = blockIdx.x * size_t(blockDim.x) + threadIdx.x; i <= nrows; i += stride) {
+        const off_t64 v = rp[i] + add;
+        for (uint32_t k = 0; k < ndst; ++k) d.rp[k][i] = v;
+    }
+    for (size_t j = blockIdx.x * size_t(blockDim.x) + threadIdx.x; j < nnz; j += stride) {
+        const idx_t c = ci[j];
+        for (uint32_t k = 0; k < ndst; ++k) d.ci[k][j] = c;
+    }
+}
+
 }  // namespace
 
 void validate_csr(const off_t64* rowptr, const idx_t* colidx, idx_t nrows, idx_t ncols, uint64_t nnz) {
@@ -216,6 +239,25 @@ void matrix_export_block(const Matrix* m, off_t64* rowptr_out, idx_t* colidx_out
     count_launch();
     check_launch("shift_rowptr_kernel");
     if (m->nnz) copy_async(colidx_out, m->colidx, m->nnz * sizeof(idx_t), cudaMemcpyDeviceToDevice);
+}
+
+// matrix_export_block to ndst destination pairs in one pass (loads once,
+// stores ndst times); ndst > kMaxPeerDst is split into launches.
+void matrix_export_block_multi(const Matrix* m, off_t64* const* rowptr_out, idx_t* const* colidx_out, uint32_t ndst,
+                               off_t64 offset) {
+    for (uint32_t k0 = 0; k0 < ndst; k0 += kMaxPeerDst) {
+        PeerDst d{};
+        const uint32_t nd = std::min<uint32_t>(kMaxPeerDst, ndst - k0);
+        for (uint32_t k = 0; k < nd; ++k) {
+            d.rp[k] = rowptr_out[k0 + k];
+            d.ci[k] = colidx_out[k0 + k];
+        }
+        const uint64_t work = std::max<uint64_t>(uint64_t(m->nrows) + 1, m->nnz);
+        export_multi_kernel<<<grid_for(work, 256), 256, 0, ctx().stream>>>(m->rowptr, m->nrows, m->colidx, m->nnz,
+                                                                          offset, d, nd);
+        count_launch();
+        check_launch("export_multi_kernel");
+    }
 }
 
 void matrix_assemble(Matrix* m, uint32_t nblocks, const idx_t* nrows, const off_t64* const* rowptr,

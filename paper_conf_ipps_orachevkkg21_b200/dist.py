@@ -78,11 +78,100 @@ def allgather_rows(ops, M_local, nrows_total, ncols, group=None):
     return ops.wrap(nrows_total, ncols, rp_all, ci_all, total)
 
 
-class CudaOps:
-    """Local operations on the CUDA library (production path)."""
+class PeerGather:
+    """All-gather of CSR row blocks by pushing over peer memory:
+    every rank holds two pairs of gathered buffers (rowptr, colidx; double
+    buffered so a push never lands in a buffer a peer may still be reading),
+    maps every other rank's buffers into its address space once (CUDA IPC
+    through torch's tensor sharing), and each step writes its own block into
+    its slice of EVERY rank's current buffer with one kernel
+    (``spbla_Matrix_ExportRowBlockMulti``: the block is loaded once and stored
+    world times -- on an NVSwitch box the peer stores go over NVLink), then
+    synchronises the device and meets the other ranks at a barrier.  No
+    collective library moves the data; NCCL/gloo only carry the block sizes,
+    the one-off IPC handles and the barrier.
 
-    def __init__(self, sp):
+    ``ok`` is False when the mapping failed on any rank (no peer access): the
+    caller then uses the broadcast all-gather."""
+
+    def __init__(self, group=None):
+        self.group = group
+        self.cap = (0, 0)
+        self.own = None
+        self.peers = None
+        self.parity = 0
+        self.ok = True
+
+    def _alloc(self, rows_cap, nnz_cap, dev):
+        from torch.multiprocessing.reductions import reduce_tensor
+        world = dist.get_world_size(self.group)
+        rank = dist.get_rank(self.group)
+        own = [(torch.empty(rows_cap, dtype=torch.int64, device=dev),
+                torch.empty(nnz_cap, dtype=torch.int32, device=dev)) for _ in range(2)]
+        mine = [[reduce_tensor(t) for t in pair] for pair in own]
+        objs = [None] * world
+        dist.all_gather_object(objs, mine, group=self.group)
+        peers, ok = [], True
+        try:
+            for b in range(world):
+                if b == rank:
+                    peers.append(own)
+                else:
+                    peers.append([tuple(fn(*args) for fn, args in pair) for pair in objs[b]])
+        except Exception:  # (no CUDA IPC / peer access between these GPUs)
+            ok = False
+        dev_flag = "cpu" if dist.get_backend(self.group) == "gloo" else dev
+        flag = torch.tensor([0 if ok else 1], dtype=torch.int64, device=dev_flag)
+        dist.all_reduce(flag, group=self.group)
+        self.ok = int(flag) == 0
+        self.own, self.peers, self.cap = own, (peers if self.ok else None), (rows_cap, nnz_cap)
+
+    def gather(self, ops, M_local, nrows_total, ncols):
+        world = dist.get_world_size(self.group)
+        rank = dist.get_rank(self.group)
+        nrows, nnz = ops.shape_nnz(M_local)
+        dev = ops.device(M_local)
+        sdev = "cpu" if dist.get_backend(self.group) == "gloo" else dev
+        sizes = torch.tensor([nrows, nnz], dtype=torch.int64, device=sdev)
+        all_sizes = [torch.empty_like(sizes) for _ in range(world)]
+        dist.all_gather(all_sizes, sizes, group=self.group)
+        all_sizes = [tuple(int(v) for v in t.cpu()) for t in all_sizes]
+        assert sum(s[0] for s in all_sizes) == nrows_total, "row blocks do not cover the matrix"
+        total = sum(s[1] for s in all_sizes)
+        rbase = [0] * world
+        nbase = [0] * world
+        for b in range(1, world):
+            rbase[b] = rbase[b - 1] + all_sizes[b - 1][0]
+            nbase[b] = nbase[b - 1] + all_sizes[b - 1][1]
+        if nrows_total + 1 > self.cap[0] or max(total, 1) > self.cap[1]:
+            # (every rank sees the same sizes: a collective decision; the
+            # closure's growing C gets 1.5x headroom)
+            self._alloc(nrows_total + 1, max(int(total * 1.5), total, 1), dev)
+            if not self.ok:
+                return None
+        p = self.parity
+        self.parity ^= 1
+        dsts = [(self.peers[b][p][0][rbase[rank]:rbase[rank] + nrows + 1],
+                 self.peers[b][p][1][nbase[rank]:nbase[rank] + max(nnz, 1)]) for b in range(world)]
+        ops.export_block_multi(M_local, dsts, nbase[rank])
+        torch.cuda.synchronize(dev)
+        dist.barrier(group=self.group)
+        rp, ci = self.own[p]
+        return ops.wrap(nrows_total, ncols, rp[:nrows_total + 1], ci[:max(total, 1)], total)
+
+
+class CudaOps:
+    """Local operations on the CUDA library (production path).  peer=True:
+    B is all-gathered by pushing over peer memory (:class:`PeerGather`),
+    falling back to the broadcast all-gather when the ranks cannot map each
+    other's memory."""
+
+    def __init__(self, sp, peer=True):
         self.sp = sp
+        self.peer = PeerGather() if peer else None
+
+    def export_block_multi(self, M, dsts, offset):
+        M.export_row_block_multi(dsts, offset)
 
     def shape_nnz(self, M):
         return M.nrows, M.nvals
@@ -115,6 +204,11 @@ def allreduce_int(x: int, group=None, op=dist.ReduceOp.SUM, device=None) -> int:
 
 
 def gather_rows(ops, M_local, nrows_total, ncols, group=None):
+    peer = getattr(ops, "peer", None)
+    if peer is not None and peer.ok and group is None:
+        B = peer.gather(ops, M_local, nrows_total, ncols)
+        if B is not None:
+            return B
     return allgather_rows(ops, M_local, nrows_total, ncols, group)
 
 

@@ -2,7 +2,8 @@
 ``spbla_Matrix_AssembleRowBlocks`` bit-exact round trip, and the
 row-partitioned ``distributed_mxm`` / ``distributed_closure`` of dist.py with
 :class:`CudaOps` at world_size 2 (two processes sharing cuda:0, gloo for the
-collectives), every rank's rows compared with the oracle."""
+collectives), with B all-gathered either by the peer-memory push kernel or by
+broadcasts, every rank's rows compared with the oracle."""
 import os
 import socket
 
@@ -53,7 +54,7 @@ def free_port():
     return p
 
 
-def worker(rank, world, port, q):
+def worker(rank, world, port, q, peer):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     import sys
@@ -65,7 +66,7 @@ def worker(rank, world, port, q):
         from paper_conf_ipps_orachevkkg21_b200 import dist as spdist
         sp.Initialize(0)
         torch.cuda.set_device(0)
-        ops = spdist.CudaOps(sp)
+        ops = spdist.CudaOps(sp, peer=peer)
         n = 1 << 13
         r, c = spgen.rmat_pairs(13, 12, 0.45, 0.22, 0.22, seed=3)
         O = oracle.build(n, n, r.numpy(), c.numpy())
@@ -97,24 +98,30 @@ def worker(rank, world, port, q):
         rp2, ci2 = Cl2.to_csr()
         want2 = rows_of(ref, s0, s1)
         ok_clo = np.array_equal(rp2, want2.rowptr) and np.array_equal(ci2, want2.colidx) and it == ref_it
-        q.put((rank, bool(ok_mxm), bool(ok_clo), it, ref_it, None))
+        used_peer = ops.peer is not None and ops.peer.ok and ops.peer.own is not None
+        q.put((rank, bool(ok_mxm), bool(ok_clo), it, ref_it, None, used_peer))
     except Exception as e:  # pragma: no cover - reported to the parent
-        q.put((rank, False, False, 0, 0, repr(e)))
+        q.put((rank, False, False, 0, 0, repr(e), False))
     finally:
         dist.destroy_process_group()
 
 
-def test_distributed_cuda_ws2():
+@pytest.mark.parametrize("peer", [True, False], ids=["peer_push", "broadcast"])
+def test_distributed_cuda_ws2(peer):
+    """peer_push: B all-gathered by the push kernel over peer memory (CUDA IPC
+    between the two processes; on one GPU the mapping is same-device);
+    broadcast: one NCCL/gloo broadcast per rank."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()
-    procs = [ctx.Process(target=worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=worker, args=(r, 2, port, q, peer)) for r in range(2)]
     for p in procs:
         p.start()
     res = [q.get(timeout=300) for _ in procs]
     for p in procs:
         p.join(timeout=60)
-    for rank, ok_mxm, ok_clo, it, ref_it, err in res:
+    for rank, ok_mxm, ok_clo, it, ref_it, err, used_peer in res:
         assert err is None, f"rank {rank}: {err}"
+        assert used_peer == peer, f"rank {rank}: peer push used = {used_peer}"
         assert ok_mxm, f"rank {rank}: distributed MxM rows differ"
         assert ok_clo, f"rank {rank}: distributed closure differs ({it} vs {ref_it} iterations)"
