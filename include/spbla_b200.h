@@ -188,6 +188,22 @@ spbla_Status spbla_Matrix_ExportRowBlock(spbla_Matrix matrix, spbla_Offset* rowp
  * destination owners read.  Errors: null matrix, null arrays or entries. */
 spbla_Status spbla_Matrix_ExportRowBlockMulti(spbla_Matrix matrix, spbla_Offset* const* rowptrs,
                                              spbla_Index* const* colidxs, uint32_t ndst, spbla_Offset offset);
+/* Peer buffers for the push all-gather: device memory of the
+ * library's GPU that other processes map through CUDA IPC.
+ * PeerBufferCreate: cudaMalloc of `bytes` (not the pools: IPC needs a whole
+ * allocation), *ptr its device address, `handle` receives the
+ * SPBLA_PEER_HANDLE_BYTES-byte IPC handle (plain bytes, for any transport).
+ * PeerBufferOpen: maps another process's buffer from its handle for the
+ * library's device (peer access enabled as needed); DEVICE_ERROR when the
+ * GPUs cannot reach each other -- the caller falls back to broadcasts.
+ * PeerBufferClose unmaps (PeerBufferOpen's pointer), PeerBufferFree frees
+ * (PeerBufferCreate's pointer, after a device synchronisation); the owner
+ * frees only after every peer has closed its mapping. */
+#define SPBLA_PEER_HANDLE_BYTES 64
+spbla_Status spbla_PeerBufferCreate(uint64_t bytes, void** ptr, void* handle);
+spbla_Status spbla_PeerBufferOpen(const void* handle, void** ptr);
+spbla_Status spbla_PeerBufferClose(void* ptr);
+spbla_Status spbla_PeerBufferFree(void* ptr);
 /* Concatenate row blocks (block b: nrows[b] rows, device arrays rowptr[b]
  * starting at 0 and colidx[b] with nnz[b] values) into `matrix` (replaced;
  * its ncols is kept; sum nrows[b] must equal its nrows).  Used to assemble a

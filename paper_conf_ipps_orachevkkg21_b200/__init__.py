@@ -130,6 +130,45 @@ def set_out_of_place_compaction(enable: bool = True):
     _check(_lib().spbla_SetOutOfPlaceCompaction(int(bool(enable))), "spbla_SetOutOfPlaceCompaction")
 
 
+PEER_HANDLE_BYTES = 64
+
+
+class PeerBuffer:
+    """Device memory that other processes map through CUDA IPC
+    (spbla_PeerBufferCreate / Open / Close / Free): the gathered buffers of
+    the push all-gather (dist.PeerGather)."""
+
+    def __init__(self, nbytes: int = 0, handle: bytes = None):
+        self.ptr, self.owner = 0, handle is None
+        p = ctypes.c_void_p()
+        if handle is None:
+            h = ctypes.create_string_buffer(PEER_HANDLE_BYTES)
+            _check(_lib().spbla_PeerBufferCreate(int(nbytes), ctypes.byref(p), h), "spbla_PeerBufferCreate")
+            self.handle = h.raw
+        else:
+            h = ctypes.create_string_buffer(bytes(handle), PEER_HANDLE_BYTES)
+            _check(_lib().spbla_PeerBufferOpen(h, ctypes.byref(p)), "spbla_PeerBufferOpen")
+            self.handle = bytes(handle)
+        self.ptr = int(p.value or 0)
+
+    def tensor(self, dtype, n: int):
+        """torch view of the first n elements (owner's buffer, this device)."""
+        import torch
+        ts = {torch.int64: "<i8", torch.int32: "<i4"}[dtype]
+
+        class _Cai:
+            def __init__(self, ptr, n, typestr):
+                self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False),
+                                                 "version": 3, "strides": None}
+        return torch.as_tensor(_Cai(self.ptr, n, ts), device=f"cuda:{_device}")
+
+    def close(self):
+        if self.ptr:
+            fn = _lib().spbla_PeerBufferFree if self.owner else _lib().spbla_PeerBufferClose
+            _check(fn(ctypes.c_void_p(self.ptr)), "spbla_PeerBufferFree/Close")
+        self.ptr = 0
+
+
 def _ptr(a):
     """Raw address of a torch tensor / numpy array, and whether it is host memory."""
     if a is None:
@@ -330,13 +369,12 @@ class Matrix:
                                                   int(offset)), "spbla_Matrix_ExportRowBlock")
 
     def export_row_block_multi(self, dsts, offset: int):
-        """export_row_block into several (rowptr, colidx) device tensor pairs
-        with one kernel (spbla_Matrix_ExportRowBlockMulti; peer-mapped
-        tensors of other ranks included)."""
+        """export_row_block into several destinations with one kernel
+        (spbla_Matrix_ExportRowBlockMulti): dsts = [(rowptr_ptr, colidx_ptr)]
+        raw device addresses -- peer-mapped buffers of other ranks included."""
         nd = len(dsts)
-        n = self.nvals
-        rps = (ctypes.c_void_p * max(nd, 1))(*[t.data_ptr() for t, _ in dsts])
-        cis = (ctypes.c_void_p * max(nd, 1))(*[(c.data_ptr() if n else 0) for _, c in dsts])
+        rps = (ctypes.c_void_p * max(nd, 1))(*[int(a) for a, _ in dsts])
+        cis = (ctypes.c_void_p * max(nd, 1))(*[int(b) for _, b in dsts])
         _check(_lib().spbla_Matrix_ExportRowBlockMulti(self._h, rps, cis, nd, int(offset)),
                "spbla_Matrix_ExportRowBlockMulti")
 

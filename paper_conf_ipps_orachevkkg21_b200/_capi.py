@@ -47,6 +47,10 @@ SIGNATURES = {
     "spbla_Matrix_DevicePointers": (_int, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp)]),
     "spbla_Matrix_ExportRowBlock": (_int, [_vp, _vp, _vp, _u64]),
     "spbla_Matrix_ExportRowBlockMulti": (_int, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _u32, _u64]),
+    "spbla_PeerBufferCreate": (_int, [_u64, ctypes.POINTER(_vp), _vp]),
+    "spbla_PeerBufferOpen": (_int, [_vp, ctypes.POINTER(_vp)]),
+    "spbla_PeerBufferClose": (_int, [_vp]),
+    "spbla_PeerBufferFree": (_int, [_vp]),
     "spbla_Matrix_AssembleRowBlocks": (_int, [_vp, _u32, _pu32, ctypes.POINTER(_vp), ctypes.POINTER(_vp), _pu64]),
     "spbla_MxM": (_int, [_vp, _vp, _vp, _u32]),
     "spbla_Matrix_EWiseAdd": (_int, [_vp, _vp, _vp, _u32]),

@@ -2,6 +2,8 @@
 // status translation around the device implementations.
 #include "common.cuh"
 
+#include <cstring>
+
 #include <cstdio>
 #include <new>
 #include <string>
@@ -299,6 +301,58 @@ spbla_Status spbla_Matrix_ExportRowBlockMulti(spbla_Matrix m, spbla_Offset* cons
         NEED(m && (ndst == 0 || (rowptrs && colidxs)), "null argument");
         for (uint32_t k = 0; k < ndst; ++k) NEED(rowptrs[k] && (m->nnz == 0 || colidxs[k]), "null destination");
         if (ndst) matrix_export_block_multi(m, rowptrs, colidxs, ndst, offset);
+    });
+}
+
+spbla_Status spbla_PeerBufferCreate(uint64_t bytes, void** ptr, void* handle) {
+    return guarded([&] {
+        require_init();
+        NEED(ptr && handle && bytes, "null argument or zero size");
+        void* p = nullptr;
+        CUDA_CHECK(cudaMalloc(&p, bytes));
+        cudaIpcMemHandle_t h;
+        const cudaError_t e = cudaIpcGetMemHandle(&h, p);
+        if (e != cudaSuccess) {
+            (void)cudaGetLastError();
+            cudaFree(p);
+            SPBLA_THROW(SPBLA_STATUS_DEVICE_ERROR, "cudaIpcGetMemHandle failed");
+        }
+        static_assert(sizeof(h) == SPBLA_PEER_HANDLE_BYTES, "IPC handle size");
+        std::memcpy(handle, &h, sizeof(h));
+        *ptr = p;
+    });
+}
+
+spbla_Status spbla_PeerBufferOpen(const void* handle, void** ptr) {
+    return guarded([&] {
+        require_init();
+        NEED(ptr && handle, "null argument");
+        cudaIpcMemHandle_t h;
+        std::memcpy(&h, handle, sizeof(h));
+        void* p = nullptr;
+        // mapped for the library's device; peer access to the owner's GPU is
+        // enabled as needed (fails cleanly when the GPUs cannot reach each other)
+        const cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+            (void)cudaGetLastError();
+            SPBLA_THROW(SPBLA_STATUS_DEVICE_ERROR, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+        }
+        *ptr = p;
+    });
+}
+
+spbla_Status spbla_PeerBufferClose(void* ptr) {
+    return guarded([&] {
+        if (ptr) CUDA_CHECK(cudaIpcCloseMemHandle(ptr));
+    });
+}
+
+spbla_Status spbla_PeerBufferFree(void* ptr) {
+    return guarded([&] {
+        if (ptr) {
+            CUDA_CHECK(cudaDeviceSynchronize());  // (peers may be mid-write only outside the protocol)
+            CUDA_CHECK(cudaFree(ptr));
+        }
     });
 }
 

@@ -81,50 +81,71 @@ def allgather_rows(ops, M_local, nrows_total, ncols, group=None):
 class PeerGather:
     """All-gather of CSR row blocks by pushing over peer memory:
     every rank holds two pairs of gathered buffers (rowptr, colidx; double
-    buffered so a push never lands in a buffer a peer may still be reading),
-    maps every other rank's buffers into its address space once (CUDA IPC
-    through torch's tensor sharing), and each step writes its own block into
-    its slice of EVERY rank's current buffer with one kernel
+    buffered so a push never lands in a buffer a peer may still be reading)
+    allocated by the library as IPC-shareable device memory, maps every other
+    rank's buffers into its address space once (CUDA IPC, opened for its own
+    GPU with peer access enabled as needed), and each step writes its own block
+    into its slice of EVERY rank's current buffer with one kernel
     (``spbla_Matrix_ExportRowBlockMulti``: the block is loaded once and stored
     world times -- on an NVSwitch box the peer stores go over NVLink), then
     synchronises the device and meets the other ranks at a barrier.  No
     collective library moves the data; NCCL/gloo only carry the block sizes,
-    the one-off IPC handles and the barrier.
+    the one-off 64-byte IPC handles and the barrier.
 
-    ``ok`` is False when the mapping failed on any rank (no peer access): the
-    caller then uses the broadcast all-gather."""
+    ``ok`` becomes False (on every rank: an all-reduced flag) when any rank
+    cannot map another's buffers; the caller then uses the broadcast
+    all-gather."""
 
-    def __init__(self, group=None):
+    def __init__(self, sp, group=None):
+        self.sp = sp
         self.group = group
         self.cap = (0, 0)
-        self.own = None
-        self.peers = None
+        self.own = None    # [parity] -> (PeerBuffer rowptr, PeerBuffer colidx)
+        self.peers = None  # [rank][parity] -> (rowptr address, colidx address)
+        self.mapped = []
         self.parity = 0
         self.ok = True
 
-    def _alloc(self, rows_cap, nnz_cap, dev):
-        from torch.multiprocessing.reductions import reduce_tensor
+    def _release(self):
+        for m in self.mapped:  # unmap the peers' buffers, then (after every
+            m.close()          # rank has) free our own
+        self.mapped = []
+        if self.own is not None:
+            dist.barrier(group=self.group)
+            for pair in self.own:
+                for buf in pair:
+                    buf.close()
+        self.own = self.peers = None
+
+    def _alloc(self, rows_cap, nnz_cap):
         world = dist.get_world_size(self.group)
         rank = dist.get_rank(self.group)
-        own = [(torch.empty(rows_cap, dtype=torch.int64, device=dev),
-                torch.empty(nnz_cap, dtype=torch.int32, device=dev)) for _ in range(2)]
-        mine = [[reduce_tensor(t) for t in pair] for pair in own]
+        self._release()
+        own = [(self.sp.PeerBuffer(rows_cap * 8), self.sp.PeerBuffer(nnz_cap * 4)) for _ in range(2)]
         objs = [None] * world
-        dist.all_gather_object(objs, mine, group=self.group)
+        dist.all_gather_object(objs, [[b.handle for b in pair] for pair in own], group=self.group)
         peers, ok = [], True
-        try:
-            for b in range(world):
-                if b == rank:
-                    peers.append(own)
-                else:
-                    peers.append([tuple(fn(*args) for fn, args in pair) for pair in objs[b]])
-        except Exception:  # (no CUDA IPC / peer access between these GPUs)
-            ok = False
-        dev_flag = "cpu" if dist.get_backend(self.group) == "gloo" else dev
+        for b in range(world):
+            if b == rank:
+                peers.append([(rp.ptr, ci.ptr) for rp, ci in own])
+                continue
+            try:
+                pair_ptrs = []
+                for hrp, hci in objs[b]:
+                    mrp, mci = self.sp.PeerBuffer(handle=hrp), self.sp.PeerBuffer(handle=hci)
+                    self.mapped += [mrp, mci]
+                    pair_ptrs.append((mrp.ptr, mci.ptr))
+                peers.append(pair_ptrs)
+            except Exception:  # (the GPUs cannot reach each other)
+                ok = False
+                break
+        dev_flag = "cpu" if dist.get_backend(self.group) == "gloo" else "cuda"
         flag = torch.tensor([0 if ok else 1], dtype=torch.int64, device=dev_flag)
         dist.all_reduce(flag, group=self.group)
+        self.own, self.peers, self.cap = own, peers, (rows_cap, nnz_cap)
         self.ok = int(flag) == 0
-        self.own, self.peers, self.cap = own, (peers if self.ok else None), (rows_cap, nnz_cap)
+        if not self.ok:
+            self._release()
 
     def gather(self, ops, M_local, nrows_total, ncols):
         world = dist.get_world_size(self.group)
@@ -146,18 +167,19 @@ class PeerGather:
         if nrows_total + 1 > self.cap[0] or max(total, 1) > self.cap[1]:
             # (every rank sees the same sizes: a collective decision; the
             # closure's growing C gets 1.5x headroom)
-            self._alloc(nrows_total + 1, max(int(total * 1.5), total, 1), dev)
+            self._alloc(nrows_total + 1, max(int(total * 1.5), total, 1))
             if not self.ok:
                 return None
         p = self.parity
         self.parity ^= 1
-        dsts = [(self.peers[b][p][0][rbase[rank]:rbase[rank] + nrows + 1],
-                 self.peers[b][p][1][nbase[rank]:nbase[rank] + max(nnz, 1)]) for b in range(world)]
+        dsts = [(self.peers[b][p][0] + 8 * rbase[rank], self.peers[b][p][1] + 4 * nbase[rank])
+                for b in range(world)]
         ops.export_block_multi(M_local, dsts, nbase[rank])
         torch.cuda.synchronize(dev)
         dist.barrier(group=self.group)
         rp, ci = self.own[p]
-        return ops.wrap(nrows_total, ncols, rp[:nrows_total + 1], ci[:max(total, 1)], total)
+        return ops.wrap(nrows_total, ncols, rp.tensor(torch.int64, nrows_total + 1),
+                        ci.tensor(torch.int32, max(total, 1)), total)
 
 
 class CudaOps:
@@ -168,7 +190,7 @@ class CudaOps:
 
     def __init__(self, sp, peer=True):
         self.sp = sp
-        self.peer = PeerGather() if peer else None
+        self.peer = PeerGather(sp) if peer else None
 
     def export_block_multi(self, M, dsts, offset):
         M.export_row_block_multi(dsts, offset)

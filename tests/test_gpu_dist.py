@@ -99,6 +99,8 @@ def worker(rank, world, port, q, peer):
         want2 = rows_of(ref, s0, s1)
         ok_clo = np.array_equal(rp2, want2.rowptr) and np.array_equal(ci2, want2.colidx) and it == ref_it
         used_peer = ops.peer is not None and ops.peer.ok and ops.peer.own is not None
+        if ops.peer is not None:
+            ops.peer._release()
         q.put((rank, bool(ok_mxm), bool(ok_clo), it, ref_it, None, used_peer))
     except Exception as e:  # pragma: no cover - reported to the parent
         q.put((rank, False, False, 0, 0, repr(e), False))
