@@ -46,6 +46,31 @@ def test_assemble_row_blocks_roundtrip():
     assert_same(sp.mxm(B, B), oracle.mxm(O, O), "A.A on the assembled matrix")
 
 
+def test_export_row_block_multi_and_peer_buffers():
+    """spbla_Matrix_ExportRowBlockMulti writes one row block (offsets shifted)
+    into many destinations at once -- 11 here, so the kernel's 8-destination
+    batches split -- including same-process IPC buffers; a garbage IPC handle
+    is a clean DEVICE_ERROR."""
+    sp = gpu_lib()
+    n = 1 << 12
+    r, c = spgen.rmat_pairs(12, 8, 0.45, 0.22, 0.22, seed=9)
+    A = sp.Matrix.from_pairs(n, n, r.cuda(), c.cuda())
+    rp, ci = A.device_tensors()
+    off = 12345
+    dsts = [(torch.zeros(n + 1, dtype=torch.int64, device="cuda"), torch.zeros(A.nvals, dtype=torch.int32, device="cuda"))
+            for _ in range(10)]
+    pb_rp, pb_ci = sp.PeerBuffer((n + 1) * 8), sp.PeerBuffer(A.nvals * 4)
+    ptrs = [(a.data_ptr(), b.data_ptr()) for a, b in dsts] + [(pb_rp.ptr, pb_ci.ptr)]
+    A.export_row_block_multi(ptrs, off)
+    torch.cuda.synchronize()
+    for a, b in dsts + [(pb_rp.tensor(torch.int64, n + 1), pb_ci.tensor(torch.int32, A.nvals))]:
+        assert torch.equal(a, rp + off) and torch.equal(b, ci)
+    pb_rp.close()
+    pb_ci.close()
+    with pytest.raises(sp.SpblaError):
+        sp.PeerBuffer(handle=bytes(64))
+
+
 def free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
