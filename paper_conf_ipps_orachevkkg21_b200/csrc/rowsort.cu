@@ -78,6 +78,9 @@ constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 #endif
 constexpr uint64_t kHB[7] = {SPBLA_HB};
 constexpr uint64_t kH0 = kHB[0], kH1 = kHB[1], kH2 = kHB[2], kH3 = kHB[3], kH4 = kHB[4], kH5 = kHB[5], kH6 = kHB[6];
+#ifndef SPBLA_PART_MIN  // partition-by-window above this many windows (overridable for a sweep)
+#define SPBLA_PART_MIN 3
+#endif
 constexpr uint32_t kDenseBits = 3u << 19;      // bitmap window: 1.5 Mi columns, 192 KB of smem
 constexpr int kUnroll = 4;                     // warp_flat (warp bins)
 
@@ -1039,7 +1042,7 @@ dense_bin_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* 
         // products), so it never overwrites an unread slice.  Two gathers
         // and a slice pass per row, whatever the number of windows.
         const uint64_t prods = ub[r] & kUbValue;
-        const bool part = nwin > 3 && prods <= soff[r + 1] - soff[r] && nwin < 2 * BATCH;
+        const bool part = nwin > SPBLA_PART_MIN && prods <= soff[r + 1] - soff[r] && nwin < 2 * BATCH;
         uint32_t* wcur = bm;               // (partition mode, during the gathers) per-window cursors
         uint32_t* wbeg = bm + kWords / 2;  // ... and slice starts (nwin + 1 entries)
         uint32_t* slb = reinterpret_cast<uint32_t*>(sd_ptr);  // slice bounds while the windows run
