@@ -1663,7 +1663,7 @@ HBIN(H4, H4_CFG)
 #endif
 HBIN(H5, H5_CFG)
 #ifndef H6_CFG  // (overridable for tools/sweep.sh)
-#define H6_CFG 1024, kH6, 192, 96, 384, 1, 6, true
+#define H6_CFG 1024, kH6, 192, 96, 384, 1, 6, false
 #endif
 HBIN(H6, H6_CFG)
 #define HASHK(N, KIND) hash_bin_kernel<N##_T, N##_B, N##_OVCAP, N##_OBCAP, N##_BATCH, N##_PERSM, N##_U, N##_DB, KIND>
