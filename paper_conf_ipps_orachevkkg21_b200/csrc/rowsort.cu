@@ -78,6 +78,9 @@ constexpr uint64_t kWarpMaxUb = kRangeMinUb;   // 256
 #endif
 constexpr uint64_t kHB[7] = {SPBLA_HB};
 constexpr uint64_t kH0 = kHB[0], kH1 = kHB[1], kH2 = kHB[2], kH3 = kHB[3], kH4 = kHB[4], kH5 = kHB[5], kH6 = kHB[6];
+#ifndef SPBLA_EARLY_STOP_MAX  // early stop in the hash bins of at most this many threads (sweeps)
+#define SPBLA_EARLY_STOP_MAX 128
+#endif
 #ifndef SPBLA_PART_MIN  // partition-by-window above this many windows (overridable for a sweep)
 #define SPBLA_PART_MIN 3
 #endif
@@ -534,7 +537,7 @@ hash_bin_kernel(SegSource src, const RowRec* __restrict__ recs, const uint32_t* 
     __shared__ uint32_t s_flag, s_novf, s_nob, s_pool;
     // early stop of the gather once the row is bound for the fallback: the
     // small bins, where duplicate-heavy closure rows overflow
-    constexpr bool kEarlyStop = THREADS <= 128;
+    constexpr bool kEarlyStop = THREADS <= SPBLA_EARLY_STOP_MAX;
     __shared__ RowPlan s_plan[2];
     const unsigned lane = lane_id(), wib = threadIdx.x >> 5;
     const uint32_t lt = (1u << lane) - 1u;
