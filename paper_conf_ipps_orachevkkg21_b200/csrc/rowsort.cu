@@ -8,7 +8,7 @@
 // Pipeline (all on the device; two host read-backs for allocation sizes):
 //   1. bin_count   : cap[r] = min(ub[r], ncols), bin[r] by ub, bin histogram
 //   2. scan(cap)   : scratch offsets (in-house decoupled look-back scan)
-//   3. bin_scatter : row lists per bin; make_recs: 40-B work records of the
+//   3. bin_scatter : row lists per bin and the 40-B work records of the
 //                    hash-bin rows
 //   4. per-bin kernels (heaviest first, persistent grids):
 //        dense (ub > 40960): one-level smem bitmap over 1.5 Mi-column
@@ -432,7 +432,7 @@ __device__ __forceinline__ void push_fallback(idx_t r, uint32_t span_m1, idx_t* 
     else ovf_rows[atomicAdd(ovf_cnt + 3, 1u)] = r;
 }
 
-// Per-row work record of the hash bins (written by make_recs_kernel after
+// Per-row work record of the hash bins (written by bin_scatter_kernel while
 // binning): one 40-B load gives everything the row needs.
 struct RowRec {
     uint32_t r, u, clo, chi;  // row, upper bound, column span [clo, chi]
@@ -1237,8 +1237,35 @@ __global__ void bin_offsets_kernel(const uint32_t* hist, uint32_t* binoff, uint3
     }
 }
 
+// The hash bins' 40-B work record of row r (row, ub, span, scratch offset,
+// descriptor base, segment count).
+__device__ __forceinline__ RowRec make_rec(const SegSource& src, idx_t r, const uint64_t* __restrict__ ub,
+                                          const uint2* __restrict__ range, idx_t ncols,
+                                          const uint64_t* __restrict__ soff) {
+    RowRec x;
+    x.r = r;
+    x.u = uint32_t(min(ub[r] & kUbValue, uint64_t(0xFFFFFFFFu)));
+    if (range) {
+        const uint2 rg = range[r];
+        x.clo = rg.x;
+        x.chi = rg.y;
+    } else {
+        x.clo = 0;
+        x.chi = ncols - 1;
+    }
+    x.out = soff[r];
+    x.seg = seg_base(src, r);
+    x.nseg = num_segs(src, r);
+    x.pad = 0;
+    return x;
+}
+
+// rows[] lists per bin; a hash-bin row's work record is written at its item
+// position at the same time (recs indexed by item)
 __global__ void bin_scatter_kernel(const uint8_t* __restrict__ bin, idx_t nrows,
-                                   uint32_t* __restrict__ cursor, idx_t* __restrict__ rows) {
+                                   uint32_t* __restrict__ cursor, idx_t* __restrict__ rows, SegSource src,
+                                   const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
+                                   const uint64_t* __restrict__ soff, RowRec* __restrict__ recs) {
     __shared__ uint32_t sh_cnt[kNumBins], sh_base[kNumBins];
     const size_t stride = size_t(gridDim.x) * blockDim.x;
     for (size_t r0 = blockIdx.x * size_t(blockDim.x); r0 < nrows; r0 += stride) {
@@ -1255,34 +1282,12 @@ __global__ void bin_scatter_kernel(const uint8_t* __restrict__ bin, idx_t nrows,
         if (threadIdx.x < kNumBins && sh_cnt[threadIdx.x])
             sh_base[threadIdx.x] = atomicAdd(&cursor[threadIdx.x], sh_cnt[threadIdx.x]);
         __syncthreads();
-        if (b > 0) rows[sh_base[b] + local] = idx_t(r);
-        __syncthreads();
-    }
-}
-
-// Work records of the hash-bin rows (items [binoff[BIN_H0], binoff[BIN_H6+1])).
-__global__ void make_recs_kernel(SegSource src, const idx_t* __restrict__ rows, const uint32_t* __restrict__ binoff,
-                                 const uint64_t* __restrict__ ub, const uint2* __restrict__ range, idx_t ncols,
-                                 const uint64_t* __restrict__ soff, RowRec* __restrict__ recs) {
-    const uint32_t lo = binoff[BIN_H0], hi = binoff[BIN_H6 + 1];
-    for (uint32_t i = lo + blockIdx.x * blockDim.x + threadIdx.x; i < hi; i += gridDim.x * blockDim.x) {
-        const idx_t r = rows[i];
-        RowRec x;
-        x.r = r;
-        x.u = uint32_t(min(ub[r] & kUbValue, uint64_t(0xFFFFFFFFu)));
-        if (range) {
-            const uint2 rg = range[r];
-            x.clo = rg.x;
-            x.chi = rg.y;
-        } else {
-            x.clo = 0;
-            x.chi = ncols - 1;
+        if (b > 0) {
+            const uint32_t item = sh_base[b] + local;
+            rows[item] = idx_t(r);
+            if (b >= BIN_H0 && b <= BIN_H6) recs[item] = make_rec(src, idx_t(r), ub, range, ncols, soff);
         }
-        x.out = soff[r];
-        x.seg = seg_base(src, r);
-        x.nseg = num_segs(src, r);
-        x.pad = 0;
-        recs[i] = x;
+        __syncthreads();
     }
 }
 
@@ -1749,7 +1754,8 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     bin_offsets_kernel<<<1, 32, 0, st>>>(hist, binoff, cursor);
     count_launch();
     DevBuf<idx_t> rows(nrows);
-    bin_scatter_kernel<<<gb, 256, 0, st>>>(bin.p, nrows, cursor, rows.p);
+    DevBuf<RowRec> recs(nrows);  // indexed by bin item (only hash-bin items are written)
+    bin_scatter_kernel<<<gb, 256, 0, st>>>(bin.p, nrows, cursor, rows.p, src, ub, range, ncols, soff.p, recs.p);
     count_launch();
     check_launch("bin_scatter_kernel");
     // one synchronisation: the scratch size and the bin histogram (empty bins
@@ -1767,10 +1773,7 @@ void row_engine(const SegSource& src, idx_t nrows, idx_t ncols, const uint64_t* 
     // the scratch is matrix storage: compacted in place it becomes colidx
     DevBuf<idx_t> scratch(scratch_total, kMat);
     DevBuf<idx_t> ovf_rows(2 * size_t(nrows));
-    DevBuf<RowRec> recs(nrows);  // indexed by bin item (only hash-bin items are written)
-    make_recs_kernel<<<gb, 256, 0, st>>>(src, rows.p, binoff, ub, range, ncols, soff.p, recs.p);
-    count_launch();
-    check_launch("make_recs_kernel");
+
     trace_mark("scratch alloc");
 
     // 4. per-bin kernels, heaviest first, back to back on the library stream
