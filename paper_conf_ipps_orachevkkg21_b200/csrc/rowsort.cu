@@ -163,7 +163,10 @@ __device__ __forceinline__ uint32_t warp_flat(const idx_t* p, uint32_t len, F&& 
 // written by that segment (each multiple of 2^kFirstShift lies in exactly one
 // non-empty segment); replaces the binary search of the gather.
 // Returns the number of products in the batch; ends with a barrier.
-constexpr uint32_t kFirstShift = 6;
+#ifndef SPBLA_FIRST_SHIFT  // (overridable for a sweep)
+#define SPBLA_FIRST_SHIFT 6
+#endif
+constexpr uint32_t kFirstShift = SPBLA_FIRST_SHIFT;
 // descriptor-mode segment base of row r: its descriptors are desc[seg_base + j]
 __device__ __forceinline__ uint64_t seg_base(const SegSource& s, idx_t r) {
     return s.kind == 1 ? 0 : s.dbase[r] + r;
