@@ -74,3 +74,24 @@ def test_random_kronecker(sp, seed):
     A, OA = both_from_pairs(sp, ma, na, *rand_pairs(rng, ma, na, "uniform"))
     B, OB = both_from_pairs(sp, mb, nb, *rand_pairs(rng, mb, nb, "skewed"))
     assert_same(sp.kronecker(A, B), oracle.kronecker(OA, OB), f"kron {ma}x{na} (x) {mb}x{nb}")
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_mxm_in_place_compaction(sp, seed):
+    """The same random shapes with the engine's in-place compaction (the mode
+    the library falls back to when memory is short) -- bit-exact."""
+    rng = np.random.default_rng(3000 + seed)
+    kind = ("uniform", "skewed", "dense")[seed % 3]
+    dims = [1, 33, 257, 1000, 4096]
+    m, k = (int(rng.choice(dims)) for _ in range(2))
+    n = int(rng.choice(dims + [1 << 20]))
+    A, OA = both_from_pairs(sp, m, k, *rand_pairs(rng, m, k, kind))
+    B, OB = both_from_pairs(sp, k, n, *rand_pairs(rng, k, n, kind))
+    sp.set_out_of_place_compaction(False)
+    try:
+        assert_same(sp.mxm(A, B), oracle.mxm(OA, OB), f"A.B {m}x{k}x{n} {kind} in place")
+        C, OC = both_from_pairs(sp, m, n, *rand_pairs(rng, m, n, "uniform"))
+        sp.MxM(C, A, B, accumulate=True)
+        assert_same(C, oracle.mxm(OA, OB, OC), "C += A.B in place")
+    finally:
+        sp.set_out_of_place_compaction(True)
