@@ -1557,6 +1557,16 @@ compact_inplace_kernel(idx_t* buf, idx_t* dst, const uint64_t* __restrict__ soff
             for (int k = 0; k < kCChunks; ++k) {
                 const int32_t e0 = 4 * (k * kCThreads + int32_t(threadIdx.x));
                 if (e0 + 3 < nxt) {  // the whole chunk in the current row (rows average thousands of words)
+                    // (a row whose shift is a multiple of 4 words: one 16-B
+                    // load; two aligned loads and a word select for the
+                    // others measured 1.5x slower)
+                    if (uint32_t(e0 + 3) < n && (reinterpret_cast<uintptr_t>(sp + e0) & 15) == 0) {
+                        const uint4 w = *reinterpret_cast<const uint4*>(sp + e0);
+                        v[4 * k] = w.x;
+                        v[4 * k + 1] = w.y;
+                        v[4 * k + 2] = w.z;
+                        v[4 * k + 3] = w.w;
+                    } else
 #pragma unroll
                     for (int j = 0; j < 4; ++j)
                         if (uint32_t(e0 + j) < n) v[4 * k + j] = sp[e0 + j];
