@@ -25,8 +25,10 @@
  *  - All device work is enqueued on the library stream (spbla_SetStream; the
  *    legacy default stream until set).  Entry points that must learn a result
  *    size on the host (Build, MxM, EWiseAdd, Transpose, ExtractSubMatrix,
- *    Reduce, TransitiveClosure) synchronise that stream once or twice; all
- *    others (AssembleRowBlocks included) are asynchronous.
+ *    Reduce, TransitiveClosure) synchronise that stream once or twice; the
+ *    peer-buffer calls (PeerBufferCreate/Open/Close/Free: cudaMalloc, CUDA
+ *    IPC) are synchronous; all others (AssembleRowBlocks included) are
+ *    asynchronous.
  *  - Pointer arguments flagged with SPBLA_HINT_HOST_MEMORY are host memory;
  *    otherwise they are device memory of the current device.  Caller-owned
  *    buffers stay caller-owned; matrices own their storage unless created by
